@@ -1,0 +1,478 @@
+#!/usr/bin/env python
+"""bench.py — the driver's benchmark contract for the load-balanced irregular nested loop.
+
+Default (N = 1): SpMV fp32 on R-MAT scale 22, edge factor 16 (BASELINE.json
+configs[1]), one `inl_spmv` call per step on a cached plan (degree bins built
+once, timed separately).  Prints ONE JSON line (rank 0).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--op spmv|sssp|bfs|pagerank]
+  python bench.py --impl reference ...   # the CPU oracle on the host cores (bounded sample)
+
+Under torchrun (N > 1) every rank owns a row block (inl_partition_rows) of an
+R-MAT graph whose scale grows with log2(N) so per-GPU work stays fixed (weak
+scaling); SpMV needs no collective (x replicated), SSSP/BFS/PageRank use the
+library's NCCL exchange.  Time = max over ranks of CUDA-event time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GTEPS and achieved HBM GB/s (fraction of peak) for SpMV/SSSP at 1/2/4/8 B200"
+FALLBACK_HBM = 6650.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["inl", "reference"], default="inl")
+    ap.add_argument("--op", choices=["spmv", "sssp", "bfs", "pagerank"], default="spmv")
+    ap.add_argument("--scale", type=int, default=None, help="R-MAT scale at N=1 (default per op)")
+    ap.add_argument("--edge-factor", type=int, default=16)
+    ap.add_argument("--bins", type=str, default="", help="t_thread,t_warp,t_block,grid_chunk,cta")
+    ap.add_argument("--thread-only", action="store_true", help="paper baseline T1 (no load balancing)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--iterations", type=int, default=20, help="PageRank iterations")
+    return ap.parse_args()
+
+
+DEFAULT_SCALE = {"spmv": 22, "sssp": 23, "bfs": 23, "pagerank": 25}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy r+w)"
+    return FALLBACK_HBM, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class Clocks:
+    """Samples nvidia-smi during the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.idx = index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+        time.sleep(0.3)
+        return self
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            try:
+                self.p.wait(timeout=5)
+            except Exception:
+                self.p.kill()
+
+    def summary(self):
+        try:
+            rows = [l.split(",") for l in open(self.f.name).read().strip().splitlines() if l.strip()]
+            os.unlink(self.f.name)
+        except Exception:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            r = [x.strip() for x in r]
+            try:
+                sm.append(float(r[0]))
+                smax.append(float(r[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, r[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        load = [s for s in sm if s > 0.5 * max(sm)] or sm
+        return {"sm_mhz": statistics.median(load), "sm_max_mhz": max(smax), "samples": len(sm),
+                "reasons": sorted(reasons)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+# --------------------------------------------------------------------------------------------
+# Workloads (inputs generated on the GPU by inlgen, bit-identical to the host generator)
+# --------------------------------------------------------------------------------------------
+
+def build_workload(op, scale, ef, world, rank, torch):
+    import inlgen
+    from paper_conf_icpp_liwb15_b200 import inl
+    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC}[op]
+    n = 1 << scale
+    b = inl.partition_rows(n, world)
+    g = inlgen.dev_build(scale, ef, seed=inlgen.SEED_GRAPH, flags=flags, row_begin=b[rank], row_end=b[rank + 1])
+    w = {"g": g, "bounds": b, "n": n, "flags": flags}
+    if op == "spmv":
+        w["val"] = inlgen.values_dev(g["row_ptr"], g["col_idx"], row_begin=b[rank])
+        w["x"] = inlgen.vector_dev(n)
+    elif op == "sssp":
+        w["w"] = inlgen.weights_dev(g["row_ptr"], g["col_idx"], row_begin=b[rank])
+    torch.cuda.synchronize()
+    return w
+
+
+def spmv_bytes(nnz, n_rows, n_global):
+    """Algorithmic bytes of one SpMV: col+val, int64 row_ptr, x once, y."""
+    return 8 * nnz + 8 * (n_rows + 1) + 4 * n_global + 4 * n_rows
+
+
+def pagerank_bytes_per_iter(nnz, n_rows, n_global):
+    """Per iteration: col, row_ptr, contribution gather once, outdeg, c' write."""
+    return 4 * nnz + 8 * (n_rows + 1) + 4 * n_global + 4 * n_rows + 4 * n_rows
+
+
+# --------------------------------------------------------------------------------------------
+
+def run_inl(a):
+    import torch
+    import torch.distributed as dist
+    import inlgen
+    from paper_conf_icpp_liwb15_b200 import inl
+
+    rank, world, local = dist_env()
+    if world != a.gpus:
+        raise SystemExit(f"--gpus {a.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    scale0 = a.scale or DEFAULT_SCALE[a.op]
+    scale = scale0 + int(round(math.log2(world)))  # weak scaling: fixed rows/nnz per GPU
+    stream = torch.cuda.Stream(local)
+    torch.cuda.set_stream(stream)
+    ctx = inl.Ctx(local)
+    if world > 1 or a.op != "spmv":
+        if world > 1:
+            ctx.comm_init(world, rank)
+    W = build_workload(a.op, scale, a.edge_factor, world, rank, torch)
+    g = W["g"]
+    A = inl.Csr(g["row_ptr"], g["col_idx"], g["n_global"], g["row_begin"])
+    bargs = [int(v) for v in a.bins.split(",")] if a.bins else []
+    bb = inl.bins(*bargs, flags=inl.BINS_THREAD_ONLY if a.thread_only else 0)
+    t0 = time.perf_counter()
+    plan = inl.Plan(ctx, A, bb)
+    torch.cuda.synchronize()
+    plan_ms = (time.perf_counter() - t0) * 1e3
+    info = plan.info()
+    nnz_local = A.nnz
+    peak, peak_src = peaks()
+
+    out = {}
+    if a.op == "spmv":
+        y = torch.empty(A.n_rows, device="cuda")
+        step = lambda: inl.spmv(ctx, A, W["val"], W["x"], y, plan)  # noqa: E731
+        units_local = nnz_local
+        bytes_local = spmv_bytes(nnz_local, A.n_rows, A.n_global)
+        launches_per_step = 1
+    elif a.op == "pagerank":
+        r = torch.empty(A.n_global, device="cuda")
+        step = lambda: inl.pagerank(ctx, A, g["out_degree"], r, 0.85, a.iterations, plan)  # noqa: E731
+        units_local = nnz_local * a.iterations
+        bytes_local = pagerank_bytes_per_iter(nnz_local, A.n_rows, A.n_global) * a.iterations
+        launches_per_step = 3 + 3 * a.iterations
+    else:
+        srcs = inlgen.sources(g["row_ptr"].cpu().numpy(), 8) if world == 1 else [0]
+        if world > 1:
+            src_t = torch.tensor(srcs, device="cuda")
+            dist.broadcast(src_t, 0)
+        out_arr = torch.empty(A.n_global, dtype=torch.int32, device="cuda")
+        state = {"i": 0, "last": None}
+
+        def step():
+            s = srcs[state["i"] % len(srcs)]
+            state["i"] += 1
+            if a.op == "sssp":
+                state["last"] = inl.sssp(ctx, A, W["w"], s, out_arr, plan)
+            else:
+                state["last"] = inl.bfs(ctx, A, s, out_arr, plan)
+        units_local = None
+        bytes_local = None
+        launches_per_step = None
+
+    for _ in range(max(a.warmup, 0)):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    reached = []
+    with Clocks(local) as ck:
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for _ in range(a.steps):
+            step()
+            if a.op in ("sssp", "bfs"):
+                reached.append(state["last"])
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_step = ms / a.steps
+
+    if a.op in ("sssp", "bfs"):
+        # m_reached = sum of degrees of reached vertices (directed CSR entries) per source
+        tot_edges = 0
+        for i in range(a.steps):
+            s = srcs[i % len(srcs)]
+            if a.op == "sssp":
+                inl.sssp(ctx, A, W["w"], s, out_arr, plan)
+                reached_mask = out_arr.view(torch.int32) != -1
+            else:
+                inl.bfs(ctx, A, s, out_arr, plan)
+                reached_mask = out_arr >= 0
+            deg = (g["row_ptr"][1:] - g["row_ptr"][:-1])
+            lo = g["row_begin"]
+            tot_edges += int(deg[reached_mask[lo:lo + A.n_rows]].sum().item())
+        units_local = tot_edges
+        relax = sum(r["edges_relaxed"] for r in reached)
+        bytes_local = 8 * relax + 16 * sum(r["frontier_total"] for r in reached)
+        launches_per_step = 1 + max(r["iterations"] for r in reached) * 2
+
+    if a.op in ("spmv", "pagerank"):  # per-step figures -> whole timed region
+        units_local *= a.steps
+        bytes_local *= a.steps
+    units = torch.tensor([float(units_local)], device="cuda")
+    byts = torch.tensor([float(bytes_local)], device="cuda")
+    if world > 1:
+        dist.all_reduce(units)
+        dist.all_reduce(byts)
+    units_total = float(units.item())
+    bytes_total = float(byts.item())
+    gteps = units_total / (ms * 1e-3) / 1e9
+    achieved_gbs = (bytes_total / world) / (ms * 1e-3) / 1e9  # per GPU
+
+    if rank == 0:
+        out.update({
+            "metric": METRIC, "value": round(gteps, 3), "unit": "GTEPS", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 5),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32" if a.op in ("spmv", "pagerank") else "u32",
+            "data": "synthetic (R-MAT A,B,C=.57,.19,.19, Philox seeds graph=1 val=3 x=4 w=2, generated on GPU)",
+            "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
+                                    "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
+                                    "bfs": "cfg5 BFS R-MAT symmetric"}[a.op],
+                       "op": a.op, "scale": scale, "edge_factor": a.edge_factor, "n": A.n_global,
+                       "nnz_total": int(units_total / a.steps / (a.iterations if a.op == "pagerank" else 1)) if a.op in ("spmv", "pagerank") else None,
+                       "rows_per_gpu": A.n_rows, "parallelism": f"row-blocks x{world}",
+                       "bins": info["bins"], "plan_ms": round(plan_ms, 3),
+                       "l2": "inputs larger than L2 (CSR streamed once per step; L2 is 126 MB)",
+                       "thread_only_baseline": bool(a.thread_only)},
+            "gpu_launches": (launches_per_step * a.steps) if launches_per_step else None,
+        })
+        frac = achieved_gbs / peak
+        out["roofline"] = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak, "unit": "GB/s",
+                           "frac": round(frac, 4), "peak_source": peak_src,
+                           "frac_of_8TBs": round(achieved_gbs / 8000.0, 4),
+                           "kernel": "k_gather (fused tile + grid-bin gather)" if a.op in ("spmv", "pagerank") else "k_expand",
+                           "alg_bytes_per_step_per_gpu": int(bytes_total / world / a.steps),
+                           "traffic": traffic_lookup(a.op, scale)}
+        out["plan"] = info
+    if a.op == "spmv" and not a.no_e2e:
+        e2e = e2e_spmv(a, ctx, g, W, torch, world, rank)
+        if rank == 0:
+            out["e2e"] = e2e
+    if a.op in ("sssp", "bfs") and rank == 0:
+        out["config"]["sources"] = srcs
+        out["config"]["iterations"] = [r["iterations"] for r in reached]
+        out["config"]["relaxations_per_m_reached"] = round(sum(r["edges_relaxed"] for r in reached) / max(units_total, 1), 3)
+    if rank == 0:
+        out["clocks"] = ck.summary()
+        if not a.no_cpu_baseline and world == 1:
+            out["cpu_baseline"] = cpu_baseline(a.op, g, W, a, torch)
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def traffic_lookup(op, scale):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        d = json.load(open(p))
+        v = d.get(f"{op}_s{scale}")
+        return v
+    except Exception:
+        return None
+
+
+def e2e_spmv(a, ctx, g, W, torch, world, rank):
+    """Same metric through the public API with HOST (pinned) buffers: H2D of the CSR, values and
+    x, a transient plan, the kernel, and D2H of y — all inside the timed region."""
+    import torch.distributed as dist
+    from paper_conf_icpp_liwb15_b200 import inl
+    rp = g["row_ptr"].cpu().pin_memory()
+    ci = g["col_idx"].cpu().pin_memory()
+    val = W["val"].cpu().pin_memory()
+    x = W["x"].cpu().pin_memory()
+    y = torch.empty(rp.numel() - 1, dtype=torch.float32).pin_memory()
+    A = inl.Csr(rp, ci, g["n_global"], g["row_begin"])
+    steps = max(3, min(a.steps, 10))
+    inl.spmv(ctx, A, val, x, y)  # warm-up
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        inl.spmv(ctx, A, val, x, y)  # returns after y is back on the host
+    dt = time.perf_counter() - t0
+    t = torch.tensor([dt], device="cuda")
+    nn = torch.tensor([float(ci.numel())], device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(nn)
+    dt = float(t.item())
+    h2d = rp.numel() * 8 + ci.numel() * 4 + val.numel() * 4 + x.numel() * 4
+    return {"value": round(float(nn.item()) * steps / dt / 1e9, 4), "unit": "GTEPS",
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(y.numel() * 4),
+            "ms_per_step": round(dt / steps * 1e3, 3), "steps": steps,
+            "path": "inl_spmv(host pinned buffers, plan=NULL): H2D + binning + gather + D2H (wall clock, synchronous)"}
+
+
+def cpu_baseline(op, g, W, a, torch, budget_s=10.0):
+    """The oracle as it stands (single thread, fp64) on the host cores, bounded sample."""
+    import oracle
+    rp = g["row_ptr"].cpu().numpy()
+    ci = g["col_idx"].cpu().numpy()
+    if op == "spmv":
+        val, x = W["val"].cpu().numpy(), W["x"].cpu().numpy()
+        reps, t0 = 0, time.perf_counter()
+        while True:
+            oracle.spmv(rp, ci, val, x)
+            reps += 1
+            if time.perf_counter() - t0 > budget_s:
+                break
+        dt = time.perf_counter() - t0
+        return {"value": round(len(ci) * reps / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                "sample": f"full cfg2 matrix ({len(ci)} nnz) x {reps} repetitions, {dt:.1f} s"}
+    if op == "pagerank":
+        t0 = time.perf_counter()
+        it = 2
+        oracle.pagerank(g["n_global"], rp, ci, g["out_degree"].cpu().numpy(), 0.85, it)
+        dt = time.perf_counter() - t0
+        return {"value": round(len(ci) * it / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                "sample": f"{it} PageRank iterations on the full graph ({len(ci)} nnz), {dt:.1f} s"}
+    import inlgen
+    src = inlgen.sources(rp, 1)[0]
+    t0 = time.perf_counter()
+    if op == "sssp":
+        d = oracle.sssp(rp, ci, W["w"].cpu().numpy().view("uint32"), src)
+        reached = d != 0xFFFFFFFF
+    else:
+        d = oracle.bfs(rp, ci, src)
+        reached = d >= 0
+    dt = time.perf_counter() - t0
+    m = int((rp[1:] - rp[:-1])[reached].sum())
+    return {"value": round(m / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"1 source ({src}), m_reached={m}, {dt:.1f} s"}
+
+
+def run_reference(a):
+    """--impl reference: the oracle (plain C, single thread) on the host cores, on this arm's
+    workload and metric.  Rank 0 only; other ranks exit 0 without work."""
+    rank, world, local = dist_env()
+    if rank != 0:
+        return
+    import numpy as np
+    import inlgen
+    import oracle
+    scale0 = a.scale or DEFAULT_SCALE[a.op]
+    scale = scale0 + int(round(math.log2(max(world, 1))))
+    # bounded: the host generator builds the graph for small scales; large ones use the GPU twin
+    try:
+        import torch
+        have_gpu = torch.cuda.is_available()
+    except Exception:
+        have_gpu = False
+    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC}[a.op]
+    if have_gpu:
+        g = inlgen.dev_build(scale, a.edge_factor, seed=inlgen.SEED_GRAPH, flags=flags)
+        rp, ci = g["row_ptr"].cpu().numpy(), g["col_idx"].cpu().numpy()
+        od = g["out_degree"].cpu().numpy() if g["out_degree"] is not None else None
+        n = g["n_global"]
+    else:
+        h = inlgen.host_build(scale, a.edge_factor, seed=inlgen.SEED_GRAPH, flags=flags)
+        rp, ci, od, n = h.row_ptr, h.col_idx, h.out_degree, h.n_global
+    if a.op == "spmv":
+        val = inlgen.values_host(rp, ci)
+        x = inlgen.vector_host(n)
+        fn = lambda: oracle.spmv(rp, ci, val, x)  # noqa: E731
+        units = len(ci)
+        sample = "full cfg2 SpMV per step"
+    elif a.op == "pagerank":
+        fn = lambda: oracle.pagerank(n, rp, ci, od, 0.85, 1)  # noqa: E731
+        units = len(ci)
+        sample = "1 PageRank iteration of the full graph per step"
+    else:
+        src = inlgen.sources(rp, 1)[0]
+        wts = inlgen.weights_host(rp, ci) if a.op == "sssp" else None
+        fn = (lambda: oracle.sssp(rp, ci, wts, src)) if a.op == "sssp" else (lambda: oracle.bfs(rp, ci, src))
+        d = fn()
+        reached = (d != 0xFFFFFFFF) if a.op == "sssp" else (d >= 0)
+        units = int(np.diff(rp)[reached].sum())
+        sample = f"one full {a.op} from source {src} per step"
+    for _ in range(max(a.warmup, 0)):
+        fn()
+    t0 = time.perf_counter()
+    for _ in range(a.steps):
+        fn()
+    dt = time.perf_counter() - t0
+    v = units * a.steps / dt / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": round(v, 5), "unit": "GTEPS", "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(dt / a.steps * 1e3, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64" if a.op in ("spmv", "pagerank") else "int64",
+            "data": "synthetic (same R-MAT recipe and seeds as the inl arm)",
+            "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
+                                    "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
+                                    "bfs": "cfg5 BFS R-MAT symmetric"}[a.op],
+                       "op": a.op, "scale": scale, "edge_factor": a.edge_factor, "n": int(n), "nnz_total": int(len(ci))},
+            "cpu_baseline": {"value": round(v, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": round(v, 5), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_inl(args)

@@ -1,0 +1,157 @@
+/* inl.h — C-ABI of libinl.so: the B200-native (sm_100a) hot path of
+ *   Li, Wu, Becchi, "Nested Parallelism on GPU: Exploring Parallelization
+ *   Templates for Irregular Loops and Recursive Computations", ICPP 2015
+ *   (/root/reference/PAPER.md; citations P<line>@<char offset>).
+ *
+ * The hot path is the paper's irregular nested loop (Fig. 1(a), P3@9300):
+ *     for i in outer (CSR rows / vertices):  for j < f(i) (nonzeros / edges): work(i, j)
+ * load-balanced by the degree f(i) against thresholds (lbTHRES, P5@366,
+ * P11@1197): small rows thread-mapped; larger rows deferred to warp-, block-
+ * or grid-mapped buffers (the dual-queue / delayed-buffer templates, P5@2078,
+ * P5@2721, P5@3623), instantiated for SpMV (P5@10072), SSSP (P5@10241),
+ * PageRank (P5@9262) and BFS (P5@11591).
+ *
+ * Conventions (all entry points):
+ *   - Return inl_status; nothing aborts and no C++ exception crosses the ABI.
+ *     On failure, inl_last_error(ctx) holds a message for that ctx.
+ *   - Array arguments may be DEVICE pointers (the fast path: results are
+ *     produced asynchronously on the ctx stream for SpMV/PageRank) or HOST
+ *     pointers (pageable or pinned): host inputs are copied to device scratch
+ *     owned by the ctx and host outputs copied back before the call returns
+ *     (the end-to-end path).  The caller owns every array; the library never
+ *     frees or retains caller memory and never writes inputs.
+ *   - CSR: row_ptr int64 [n_rows+1], row_ptr[0] == 0, non-decreasing;
+ *     col_idx int32 [nnz] global column ids in [0, n_global).  Contents are
+ *     not checked on the hot path (malformed CSR = undefined behaviour unless
+ *     inl_csr_validate is called).  Rows are local to a rank: global row id =
+ *     row_begin + local row (row_begin = 0, n_rows = n_global on one GPU).
+ *   - A ctx is not thread-safe; use one ctx per host thread / rank.
+ *   - Multi-GPU: every rank calls the same ops in the same order (NCCL rule);
+ *     ranks own contiguous row blocks from inl_partition_rows.
+ */
+#ifndef INL_H
+#define INL_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  INL_OK = 0,
+  INL_ERR_INVALID_ARGUMENT = 1,
+  INL_ERR_OUT_OF_MEMORY = 2,
+  INL_ERR_CUDA = 3,
+  INL_ERR_NCCL = 4,
+  INL_ERR_NOT_INITIALIZED = 5,
+  INL_ERR_UNSUPPORTED = 6,
+  INL_ERR_INTERNAL = 7
+} inl_status;
+
+typedef struct inl_ctx_s *inl_ctx;   /* device, stream, optional NCCL comm, scratch arena */
+typedef struct inl_plan_s *inl_plan; /* degree bins / work queues for one CSR on one ctx */
+
+typedef struct {
+  int64_t n_rows;         /* local rows on this rank (= n_global on one GPU) */
+  int64_t n_global;       /* global vertex / column count n */
+  int64_t row_begin;      /* global id of local row 0 (0 on one GPU) */
+  int64_t nnz;            /* local nnz = row_ptr[n_rows] */
+  const int64_t *row_ptr; /* [n_rows+1] */
+  const int32_t *col_idx; /* [nnz] */
+} inl_csr;
+
+/* Load-balancing thresholds (the paper's lbTHRES, P5@366; 0 = default).
+ * A row / vertex of degree f goes to the
+ *   thread bin  if f <= t_thread               (one lane runs the inner loop serially)
+ *   warp bin    if t_thread < f <= t_warp       (one warp, lanes stride the inner loop)
+ *   block bin   if t_warp < f <= t_block       (SpMV/PR: grid_chunk pieces, one warp each, for
+ *                                                consecutive warps; SSSP/BFS: one CTA)
+ *   grid bin    if f > t_block                 (grid_chunk-sized pieces spread over the grid)
+ * Ties go to the lower bin (reading R6 of DESIGN.md: "f(i) greater than lbTHRES
+ * is processed block-mapped", P11@1197).  t_thread = -1 means 0 (no thread bin).
+ * flags: INL_BINS_THREAD_ONLY runs the paper's baseline (thread-mapped outer loop,
+ * no load balancing, P5@14490). */
+enum { INL_BINS_THREAD_ONLY = 1 };
+typedef struct {
+  int32_t t_thread;    /* default 8 */
+  int32_t t_warp;      /* default 128, in [16, 4096] (SpMV/PR warp tiles hold < 2*t_warp nnz) */
+  int32_t t_block;     /* default 16384, >= t_warp */
+  int32_t grid_chunk;  /* default 4096 nnz per block/grid-bin piece (one warp each), in [32, 2^20] */
+  int32_t cta_threads; /* reserved (128/256/512 accepted); kernels use fixed CTA shapes */
+  int32_t flags;
+} inl_bins;
+
+typedef struct {
+  int32_t iterations;     /* frontier iterations / BFS levels executed */
+  int64_t edges_relaxed;  /* sum of the degrees of all frontier vertices expanded */
+  int64_t frontier_total; /* sum of frontier sizes over the iterations */
+} inl_stats;
+
+/* Plan summary (for tests and the bench; counts per bin). */
+typedef struct {
+  int64_t n_tiles;        /* row tiles holding the thread/warp/block-bin rows */
+  int64_t rows_thread, rows_warp, rows_block, rows_grid;
+  int64_t nnz_thread, nnz_warp, nnz_block, nnz_grid;
+  int64_t n_grid_chunks;  /* CTAs of the grid/long-row kernel */
+  inl_bins bins;          /* thresholds in effect */
+} inl_plan_info;
+
+const char *inl_version(void);
+const char *inl_status_string(inl_status s);
+const char *inl_last_error(inl_ctx ctx);
+
+/* device: CUDA ordinal; cuda_stream: cudaStream_t (NULL = legacy default stream). */
+inl_status inl_ctx_create(inl_ctx *out, int device, void *cuda_stream);
+inl_status inl_ctx_set_stream(inl_ctx ctx, void *cuda_stream);
+inl_status inl_ctx_destroy(inl_ctx ctx);
+
+/* Row-block partition (host only, no GPU needed): bounds[p] = min(p*B, n),
+ * B = ceil(n / nranks), p = 0..nranks.  Equal block sizes keep the NCCL
+ * allgather counts equal (the last block is padded). */
+inl_status inl_partition_rows(int64_t n, int32_t nranks, int64_t *bounds);
+
+/* NCCL bootstrap: rank 0 calls inl_nccl_unique_id and broadcasts the 128 bytes
+ * (torch.distributed in the Python binding); every rank then calls inl_comm_init. */
+inl_status inl_nccl_unique_id(uint8_t out[128]);
+inl_status inl_comm_init(inl_ctx ctx, const uint8_t uid[128], int32_t nranks, int32_t rank);
+
+/* Degree binning, built once and reused across calls on the
+ * same CSR (device pointers only).  bins may be NULL (defaults). */
+inl_status inl_plan_create(inl_ctx ctx, const inl_csr *A, const inl_bins *bins, inl_plan *out);
+inl_status inl_plan_get_info(inl_plan plan, inl_plan_info *info);
+inl_status inl_plan_destroy(inl_plan plan);
+
+/* O(nnz) device check of the CSR invariants (never on the hot path). */
+inl_status inl_csr_validate(inl_ctx ctx, const inl_csr *A);
+
+/* SpMV (P5@10072, P5@10497): y[i] = sum_{k in row i} val[k] * x[col_idx[k]] for the
+ * n_rows local rows; x has n_global entries.  fp32 in, fp32 accumulate, fp32 out.
+ * Each row's reduction order depends only on its degree and the bins, so y is
+ * bit-identical across partitions and runs.  plan: NULL = transient bins built
+ * inside the call (cost included), else a plan created from this same inl_csr. */
+inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y,
+                    inl_plan plan);
+
+/* PageRank (P5@9262, P5@9781; reading R1): A_in = in-edge CSR (rows =
+ * destinations, cols = sources), out_degree [n_global].  PR^0 = 1/n;
+ * PR^{t+1}(v) = (1-d)/n + d*(sum_{u->v} PR^t(u)/outdeg(u) + D^t/n), D^t = rank of
+ * dangling pages.  rank [n_global] fp32 (replicated on every rank).  damping in
+ * [0,1), iterations >= 0. */
+inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_degree, float damping,
+                        int32_t iterations, float *rank, inl_plan plan);
+
+/* SSSP (P5@10241, P11@2218): frontier Bellman-Ford relaxation (atomicMin) until
+ * no distance changes.  w [nnz] uint32 >= 1, dist [n_global] uint32 with
+ * UINT32_MAX = unreachable (replicated).  Distances must stay < 2^32 - 2^8.
+ * Blocks until converged. */
+inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source,
+                    uint32_t *dist, inl_stats *stats, inl_plan plan);
+
+/* BFS (P5@11591): level-synchronous frontier expansion; level [n_global] int32,
+ * -1 = unreachable, level[source] = 0 (replicated).  Blocks until converged. */
+inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
+                   inl_stats *stats, inl_plan plan);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,388 @@
+// frontier.cu — SSSP (PAPER.md P5@10241, P11@2218) and BFS (P5@11591) as a
+// frontier worklist over the CSR, load-balanced with the paper's delayed-buffer
+// templates:
+//   * k_expand: one thread per frontier vertex (thread-mapped outer loop).  A
+//     vertex with degree <= t_thread runs its inner loop serially in that lane;
+//     larger ones are deferred to a shared-memory buffer and processed, after
+//     __syncthreads, warp-mapped (<= t_warp) or block-mapped (<= t_block) by the
+//     same CTA (dbuf-shared, P5@3623); the largest are appended as grid_chunk
+//     chunks to a global buffer (dbuf-global, P5@2721) that k_expand_grid
+//     processes with one CTA per chunk.
+//   * SSSP relaxation: nd = dist[u] + w; atomicMin(&dist[v], nd); an improved v
+//     is claimed once per iteration (iteration stamp) and enqueued with one
+//     atomicAdd per coalesced group.  The asynchronous (single-array) variant
+//     converges to the same unique distances (reading R4).
+//   * BFS claim: atomicOr on a visited bitmap (8.4 MB at scale 26, L2-resident);
+//     the winner writes level[v] = L + 1 and enqueues v.
+//   * P > 1 ranks (row blocks): synchronous rounds; SSSP allreduce-min of dist,
+//     BFS allreduce-max of an n-byte next-frontier map, each with a
+//     trailing termination word.
+#include <cooperative_groups.h>
+
+#include "comm.h"
+#include "inl_internal.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace inl {
+
+namespace {
+
+constexpr int NT = 256;
+constexpr int NW = NT / 32;
+
+__device__ __forceinline__ void push(int32_t *q, int *cnt, int32_t v) {
+  cg::coalesced_group g = cg::coalesced_threads();
+  int pos = 0;
+  if (g.thread_rank() == 0) pos = atomicAdd(cnt, (int)g.size());
+  pos = g.shfl(pos, 0) + (int)g.thread_rank();
+  q[pos] = v;
+}
+
+struct SsspOp {
+  uint32_t *dist;       // [n_global (+1 flag word on P > 1)]
+  const uint32_t *w;    // [nnz]
+  int *stamp;           // [n_global] (!DIST)
+  uint32_t *flag;       // P > 1: dist[n] cleared on any improvement
+  int iter;
+  int64_t row_begin;
+  bool enqueue;         // !DIST: enqueue improved vertices directly
+  __device__ __forceinline__ uint32_t load(int32_t u) const {
+    return *(volatile uint32_t *)(dist + row_begin + u);
+  }
+  __device__ __forceinline__ void edge(uint32_t du, int64_t k, int32_t v, int32_t *q, int *cnt) const {
+    const uint32_t nd = du + __ldg(w + k);
+    if (nd < dist[v]) {
+      const uint32_t old = atomicMin(dist + v, nd);
+      if (nd < old) {
+        if (enqueue) {
+          if (atomicExch(stamp + v, iter) != iter) push(q, cnt, v);
+        } else {
+          *flag = 0u;
+        }
+      }
+    }
+  }
+};
+
+struct BfsOp {
+  uint32_t *bitmap;  // visited, [ceil(n/32)]
+  int32_t *level;    // [n_global]
+  uint8_t *next;     // P > 1: n-byte next map (+ flag byte at [n])
+  int64_t n;
+  int L;
+  bool enqueue;      // !DIST
+  __device__ __forceinline__ uint32_t load(int32_t) const { return 0u; }
+  __device__ __forceinline__ void edge(uint32_t, int64_t, int32_t v, int32_t *q, int *cnt) const {
+    const uint32_t bit = 1u << (v & 31);
+    if (!(bitmap[v >> 5] & bit)) {
+      if (enqueue) {
+        const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
+        if (!(old & bit)) {
+          level[v] = L + 1;
+          push(q, cnt, v);
+        }
+      } else {
+        next[v] = 1;
+        next[n] = 1;
+      }
+    }
+  }
+};
+
+struct ExpandArgs {
+  const int32_t *F;  // frontier (local row ids)
+  int nF;
+  const int64_t *rp;
+  const int32_t *col;
+  int t_thread, t_warp, t_block, chunk;
+  int2 *gitems;  // grid-bin chunk buffer
+  int *gcount;
+  int32_t *Fout;
+  int *fcount;
+  unsigned long long *relaxed;
+};
+
+template <class Op>
+__global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
+  __shared__ int32_t lw[NT], lb[NT];
+  __shared__ int nw, nb;
+  __shared__ unsigned long long red[NW];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) {
+    nw = 0;
+    nb = 0;
+  }
+  __syncthreads();
+  const int i = blockIdx.x * NT + tid;
+  unsigned long long mydeg = 0;
+  if (i < a.nF) {
+    const int32_t u = a.F[i];
+    const int64_t rs = a.rp[u], re = a.rp[u + 1];
+    const int64_t d = re - rs;
+    mydeg = (unsigned long long)d;
+    if (d <= a.t_thread) {  // thread bin: serial inner loop in this lane
+      const uint32_t su = op.load(u);
+      for (int64_t k = rs; k < re; ++k) op.edge(su, k, __ldg(a.col + k), a.Fout, a.fcount);
+    } else if (d <= a.t_warp) {
+      lw[atomicAdd(&nw, 1)] = u;
+    } else if (d <= a.t_block) {
+      lb[atomicAdd(&nb, 1)] = u;
+    } else {  // grid bin: global delayed buffer
+      const int nch = (int)((d + a.chunk - 1) / a.chunk);
+      const int base = atomicAdd(a.gcount, nch);
+      for (int c = 0; c < nch; ++c) a.gitems[base + c] = make_int2(u, c);
+    }
+  }
+  __syncthreads();
+  for (int j = warp; j < nw; j += NW) {  // warp bin
+    const int32_t u = lw[j];
+    const int64_t rs = a.rp[u], re = a.rp[u + 1];
+    const uint32_t su = op.load(u);
+    for (int64_t k = rs + lane; k < re; k += 32) op.edge(su, k, __ldg(a.col + k), a.Fout, a.fcount);
+  }
+  for (int j = 0; j < nb; ++j) {  // block bin
+    const int32_t u = lb[j];
+    const int64_t rs = a.rp[u], re = a.rp[u + 1];
+    const uint32_t su = op.load(u);
+    for (int64_t k = rs + tid; k < re; k += NT) op.edge(su, k, __ldg(a.col + k), a.Fout, a.fcount);
+  }
+  for (int o = 16; o > 0; o >>= 1) mydeg += __shfl_xor_sync(0xffffffffu, mydeg, o);
+  if (lane == 0) red[warp] = mydeg;
+  __syncthreads();
+  if (tid == 0) {
+    unsigned long long s = 0;
+    for (int q = 0; q < NW; ++q) s += red[q];
+    if (s) atomicAdd(a.relaxed, s);
+  }
+}
+
+template <class Op>
+__global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
+  const int n = *(volatile int *)a.gcount;
+  for (int it = blockIdx.x; it < n; it += gridDim.x) {
+    const int2 g = a.gitems[it];
+    const int64_t rs = a.rp[g.x], re = a.rp[g.x + 1];
+    const int64_t ks = rs + (int64_t)g.y * a.chunk;
+    const int64_t ke = min(ks + (int64_t)a.chunk, re);
+    const uint32_t su = op.load(g.x);
+    for (int64_t k = ks + threadIdx.x; k < ke; k += NT)
+      op.edge(su, k, __ldg(a.col + k), a.Fout, a.fcount);
+  }
+}
+
+__global__ void k_init_sssp(uint32_t *dist, int64_t n, int64_t s) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    dist[i] = i == s ? 0u : 0xFFFFFFFFu;
+}
+
+__global__ void k_init_bfs(int32_t *level, uint32_t *bm, int64_t n, int64_t s) {
+  const int64_t nw = (n + 31) / 32;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n || i < nw;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    if (i < n) level[i] = i == s ? 0 : -1;
+    if (i < nw) bm[i] = (i == (s >> 5)) ? (1u << (s & 31)) : 0u;
+  }
+}
+
+// P > 1: vertices of the owned slice whose distance dropped -> next frontier.
+__global__ void k_sssp_collect(const uint32_t *__restrict__ dist, uint32_t *__restrict__ prev,
+                               int64_t row_begin, int64_t n_rows, int32_t *q, int *cnt) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n_rows;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t d = dist[row_begin + v];
+    if (d < prev[v]) {
+      prev[v] = d;
+      push(q, cnt, (int32_t)v);
+    }
+  }
+}
+
+__global__ void k_copy_u32(const uint32_t *__restrict__ a, uint32_t *__restrict__ b, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    b[i] = a[i];
+}
+
+// P > 1: apply the allreduced next map: new vertices get level L+1; owned ones
+// form the next local frontier.
+__global__ void k_bfs_apply(const uint8_t *__restrict__ next, int64_t n, int32_t *level,
+                            uint32_t *bm, int L, int64_t row_begin, int64_t n_rows, int32_t *q,
+                            int *cnt) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    if (next[v] && level[v] < 0) {
+      level[v] = L + 1;
+      atomicOr(bm + (v >> 5), 1u << (v & 31));
+      if (v >= row_begin && v < row_begin + n_rows) push(q, cnt, (int32_t)(v - row_begin));
+    }
+  }
+}
+
+int grid_for(int64_t n, int sms) {
+  int64_t g = (n + 255) / 256;
+  if (g > (int64_t)sms * 16) g = (int64_t)sms * 16;
+  return g < 1 ? 1 : (int)g;
+}
+
+struct FrontierBufs {
+  int32_t *F, *Fout;
+  int2 *gitems;
+  int *counts;  // [0] fcount [1] gcount
+  unsigned long long *relaxed;
+  int *h_counts;  // pinned
+};
+
+FrontierBufs frontier_bufs(inl_ctx ctx, const inl_csr &G, const Bins &b) {
+  FrontierBufs f;
+  const int64_t n = G.n_global;
+  f.F = (int32_t *)ctx->s_a.get(sizeof(int32_t) * (n + 1));
+  f.Fout = (int32_t *)ctx->s_b.get(sizeof(int32_t) * (n + 1));
+  const int64_t mn = b.t_block < b.grid_chunk ? b.t_block : b.grid_chunk;
+  const int64_t gcap = G.nnz / (mn > 0 ? mn : 1) * 2 + 64;
+  f.gitems = (int2 *)ctx->s_c.get(sizeof(int2) * gcap);
+  f.counts = (int *)ctx->s_f.get(64);
+  f.relaxed = (unsigned long long *)(f.counts + 8);
+  f.h_counts = (int *)ctx->pinned;
+  return f;
+}
+
+template <class Op>
+void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int nF, const Op &op) {
+  cudaStream_t st = ctx->stream;
+  INL_CUDA(cudaMemsetAsync(f.counts, 0, 2 * sizeof(int), st));
+  ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, b.grid_chunk,
+               f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
+  if (nF > 0) k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
+  k_expand_grid<Op><<<ctx->num_sms * 2, NT, 0, st>>>(a, op);
+  INL_CUDA(cudaGetLastError());
+}
+
+int read_count(inl_ctx ctx, const int *d) {
+  INL_CUDA(cudaMemcpyAsync(ctx->pinned, d, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  return *(volatile int *)ctx->pinned;
+}
+
+void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_t ftotal) {
+  if (!st) return;
+  unsigned long long r = 0;
+  INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, ctx->stream));
+  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  st->iterations = iters;
+  st->edges_relaxed = (int64_t)r;
+  st->frontier_total = ftotal;
+}
+
+}  // namespace
+
+void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
+              uint32_t *dist, inl_stats *stats) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = G.n_global;
+  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  FrontierBufs f = frontier_bufs(ctx, G, b);
+  INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
+  uint32_t *D = dist;
+  uint32_t *prev = nullptr;
+  int *stamp = nullptr;
+  if (DIST) {
+    D = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * (n + 1));
+    prev = (uint32_t *)ctx->s_e.get(sizeof(uint32_t) * (G.n_rows + 1));
+  } else {
+    stamp = (int *)ctx->s_d.get(sizeof(int) * n);
+    INL_CUDA(cudaMemsetAsync(stamp, 0xFF, sizeof(int) * n, st));
+  }
+  k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(D, n, source);
+  INL_CUDA(cudaGetLastError());
+  int nF = 0;
+  const bool owned = source >= G.row_begin && source < G.row_begin + G.n_rows;
+  if (owned) {
+    const int32_t s_local = (int32_t)(source - G.row_begin);
+    INL_CUDA(cudaMemcpyAsync(f.F, &s_local, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+    nF = 1;
+  }
+  if (DIST) k_copy_u32<<<grid_for(G.n_rows, ctx->num_sms), 256, 0, st>>>(D + G.row_begin, prev, G.n_rows);
+  int iters = 0;
+  int64_t ftotal = 0;
+  for (;;) {
+    ftotal += nF;
+    if (!DIST) {
+      if (nF == 0) break;
+      SsspOp op{D, w, stamp, nullptr, iters, 0, true};
+      expand(ctx, G, b, f, nF, op);
+      ++iters;
+      nF = read_count(ctx, f.counts);
+      std::swap(f.F, f.Fout);
+    } else {
+      // flag word D[n] = 1 ("no change"), cleared by any improvement on any rank
+      const uint32_t one = 1u;
+      INL_CUDA(cudaMemcpyAsync(D + n, &one, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+      SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false};
+      expand(ctx, G, b, f, nF, op);
+      comm_allreduce(ctx, D, n + 1, ncclUint32, ncclMin);
+      ++iters;
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, D + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaStreamSynchronize(st));
+      if (*(volatile uint32_t *)ctx->pinned == 1u) break;
+      INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+      k_sssp_collect<<<grid_for(G.n_rows, ctx->num_sms), 256, 0, st>>>(D, prev, G.row_begin, G.n_rows,
+                                                                      f.F, f.counts);
+      INL_CUDA(cudaGetLastError());
+      nF = read_count(ctx, f.counts);
+    }
+  }
+  if (DIST)
+    INL_CUDA(cudaMemcpyAsync(dist, D, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, st));
+  finish_stats(ctx, f, stats, iters, ftotal);
+}
+
+void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
+             inl_stats *stats) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = G.n_global;
+  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  FrontierBufs f = frontier_bufs(ctx, G, b);
+  INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
+  uint32_t *bm = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * ((n + 31) / 32 + 1));
+  uint8_t *next = DIST ? (uint8_t *)ctx->s_e.get(n + 1) : nullptr;
+  k_init_bfs<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(level, bm, n, source);
+  INL_CUDA(cudaGetLastError());
+  int nF = 0;
+  if (source >= G.row_begin && source < G.row_begin + G.n_rows) {
+    const int32_t s_local = (int32_t)(source - G.row_begin);
+    INL_CUDA(cudaMemcpyAsync(f.F, &s_local, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+    nF = 1;
+  }
+  int L = 0;
+  int64_t ftotal = 0;
+  for (;;) {
+    ftotal += nF;
+    if (!DIST) {
+      if (nF == 0) break;
+      BfsOp op{bm, level, nullptr, n, L, true};
+      expand(ctx, G, b, f, nF, op);
+      nF = read_count(ctx, f.counts);
+      std::swap(f.F, f.Fout);
+      ++L;
+    } else {
+      INL_CUDA(cudaMemsetAsync(next, 0, n + 1, st));
+      BfsOp op{bm, level, next, n, L, false};
+      expand(ctx, G, b, f, nF, op);
+      comm_allreduce(ctx, next, n + 1, ncclUint8, ncclMax);
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, next + n, 1, cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaStreamSynchronize(st));
+      if (*(volatile uint8_t *)ctx->pinned == 0) break;
+      INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+      k_bfs_apply<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(next, n, level, bm, L, G.row_begin,
+                                                            G.n_rows, f.F, f.counts);
+      INL_CUDA(cudaGetLastError());
+      nF = read_count(ctx, f.counts);
+      ++L;
+    }
+  }
+  finish_stats(ctx, f, stats, L, ftotal);
+}
+
+}  // namespace inl

@@ -1,0 +1,398 @@
+// gather.cuh — the load-balanced irregular-nested-loop gather (SpMV, PageRank pull).
+//
+// Paper: the loop nest of Fig. 1(a) (P3@9300) — outer loop over CSR rows, inner
+// loop over the row's nonzeros — with the load-balancing templates of Fig. 1(b,c):
+// rows whose inner loop is short are thread-mapped; longer ones are deferred to a
+// buffer and processed by a wider group of threads — in the same kernel
+// (dbuf-shared, P5@3623) or spread over the grid (dbuf-global, P5@2721).
+//
+// B200 design.  Measured ceilings on B200 (scripts/microbench,
+// profiles/): streaming col_idx+val alone runs at 6.7 TB/s, but every random
+// x[col] gather costs one L1TEX wavefront per distinct 128-B line, ~1 per SM-cycle,
+// so plain gathers cap SpMV at ~230 us on R-MAT scale 22.  Hence:
+//  * HOT COLUMNS IN SHARED MEMORY: the plan ranks columns by in-degree and remaps the
+//    n_hot most frequent ones (~53% of all gathers at scale 22) to slots of a
+//    shared-memory copy of x (bank-conflict cost instead of one line per lane).
+//  * ONE CTA PER SM, 32 WARPS, and every unit of work belongs to ONE WARP — no
+//    CTA-wide barrier after the x_hot fill.  Work items (plan.cu): TILES =
+//    contiguous row ranges (<= kTileRows rows) of rows of degree <= t_warp whose
+//    nonzeros form one contiguous span (< 2*t_warp - 14 entries); CHUNKS = grid_chunk
+//    pieces of rows of degree > t_warp cut at row-relative offsets (a warp streams a
+//    chunk in passes of 2*t_warp - 32 entries).
+//  * Per item: 256-bit evict-first loads of the (remapped) col_idx and val span,
+//    the gathers (smem for hot, read-only path with L2 evict-last for cold), the
+//    products staged in a per-warp shared buffer; then THREAD bin: a lane sums its
+//    row serially (degree <= t_thread); WARP bin: rows above t_thread are deferred
+//    in a ballot mask (the shared delayed buffer of dbuf-shared, held in registers)
+//    and summed by the warp (lane stride + xor tree).  A chunk is summed by the
+//    warp; the last chunk of a row (atomic ticket) combines the partials in chunk
+//    order (fp64).  Chunked rows of degree <= t_block are the BLOCK bin (their
+//    pieces go to consecutive warps), longer ones the GRID bin.
+//  * Each row's summation order depends only on its degree and the bins — never on
+//    the tile it lands in or on alignment — so results are bit-identical across
+//    partitions (multi-GPU) and runs.  No float atomics.
+#pragma once
+#include <cuda/atomic>
+
+#include "inl_internal.cuh"
+#include "ptx.cuh"
+
+namespace inl {
+
+constexpr int kGatherWarps = 32;          // warps per CTA (1 CTA per SM)
+constexpr int kSmemBudget = 224 * 1024;   // dynamic shared memory of the gather CTA
+constexpr int kMaxHot = 32768;            // measured best x_hot size at scale 22 (128 KB)
+
+constexpr int kTileSpan = 2048;  // target nonzeros per tile (tiles hold < kTileSpan + t_warp)
+__host__ __device__ constexpr int tile_stride(int t_warp) { return kTileSpan; }
+
+// Per-warp shared scratch of a tile: the non-empty rows in order (start offset within the
+// tile span, local row id) and the row-start bitmap of the current 256-entry pass.
+struct WarpTileSmem {
+  short nzrow[kTileRows];
+};
+
+// hot slots that fit next to the per-warp tile scratch
+inline int64_t hot_capacity(int t_warp) {
+  (void)t_warp;
+  int64_t b = kSmemBudget - (int64_t)kGatherWarps * (int64_t)sizeof(WarpTileSmem) - 1024;
+  int64_t k = b / 4;
+  if (k > kMaxHot) k = kMaxHot;
+  return k < 0 ? 0 : (k & ~(int64_t)3);
+}
+
+// Epilogue for SpMV: y[r] = sum.
+struct SpmvEpi {
+  float *y;
+  static constexpr bool kDangling = false;
+  __device__ __forceinline__ void init() {}
+  __device__ __forceinline__ double operator()(int64_t r, float s) const {
+    y[r] = s;
+    return 0.0;
+  }
+};
+
+// Epilogue for one PageRank step (reading R1): PR'(v) = base + d * s(v) with
+// base = (1-d)/n + d*D/n; writes the next contribution c'(v) = PR'(v)/outdeg(v)
+// (0 for dangling pages) and, on the last step, the rank.  Returns PR'(v) for
+// dangling pages so the warp can form its fixed-order partial of D'.
+struct PrEpi {
+  const int32_t *out_degree;  // [n_global]
+  float *c_next;              // [n_global]; this rank writes its own rows
+  float *rank_out;            // [n_global] or nullptr
+  const float *base_ptr;      // device scalar
+  float damping;
+  int64_t row_begin;
+  float base;
+  static constexpr bool kDangling = true;
+  __device__ __forceinline__ void init() { base = *base_ptr; }
+  __device__ __forceinline__ double operator()(int64_t r, float s) const {
+    const int64_t v = row_begin + r;
+    const float pr = fmaf(damping, s, base);
+    const int od = __ldg(out_degree + v);
+    c_next[v] = od > 0 ? pr / (float)od : 0.0f;
+    if (rank_out) rank_out[v] = pr;
+    return od == 0 ? (double)pr : 0.0;
+  }
+};
+
+struct GatherArgs {
+  const int64_t *row_ptr;
+  const int32_t *col_idx;  // the plan's remapped copy (hot entries 0x80000000 | h)
+  const float *val;        // nullptr => implicit 1 (PageRank pull)
+  const float *x;
+  int64_t nnz, n_rows;
+  int t_thread, t_warp, t_block, chunk;
+  bool vec;  // col_idx / val 32-B aligned: 256-bit loads allowed
+};
+
+struct GatherPlan {
+  const WorkItem *items;
+  int n_items;
+  float *partials;
+  int *tickets;
+  double *dpart;        // [n_items] or nullptr
+  const float *x_hot;   // [n_hot]
+  int n_hot;
+  const uint32_t *rs_bits;  // [nnz/32 + 1] bit k set iff entry k starts a non-empty row
+};
+
+__device__ __forceinline__ float gather_x(int32_t c, const float *xs, const float *x, uint64_t polx) {
+  return c < 0 ? xs[c & 0x7fffffff] : ld_gather_f32(x + c, polx);
+}
+
+// x[c] for a remapped column: hot slots from shared memory, cold ones from global
+// (read-only path, L2 evict-last).  Branch-free.
+__device__ __forceinline__ float gx(int32_t c, bool in, const float *xs, const float *x, uint64_t polx) {
+  const bool hot = c < 0;
+  const float hv = xs[hot ? (c & 0x7fffffff) : 0];
+  const float cv = ld_gather_pred(x + (hot ? 0 : c), in && !hot, polx);
+  return hot ? hv : cv;
+}
+
+__device__ __forceinline__ float lval(const float *val, int64_t k, bool in) {
+  return val ? __uint_as_float(ld_stream_pred(val + k, in)) : (in ? 1.0f : 0.0f);
+}
+
+// L2 prefetch of entries [lo, hi) of the col/val streams (short range: one pass ahead keeps
+// the in-flight prefetch of all 4.7K warps at ~10 MB, far below the 126 MB L2).
+template <bool VALS>
+__device__ __forceinline__ void prefetch_entries(const GatherArgs &a, int64_t lo, int64_t hi) {
+  prefetch_span(a.col_idx + lo, a.col_idx + hi, a.col_idx + a.nnz);
+  if (VALS) prefetch_span(a.val + lo, a.val + hi, a.val + a.nnz);
+}
+
+template <bool VALS>
+__device__ __forceinline__ void prefetch_item(const GatherArgs &a, const WorkItem &it) {
+  prefetch_entries<VALS>(a, it.s, min(it.e, it.s + 256));
+  if (it.j < 0) prefetch_span(a.row_ptr + it.r0, a.row_ptr + it.r1 + 1, a.row_ptr + a.n_rows + 1);
+}
+
+// Stream registers of one pass: lane l holds entries q0 .. q0+7 of the item span.
+struct PassRegs {
+  uint32_t cv[8];
+  float vv[8];
+};
+
+template <bool VALS>
+__device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int len, int q0, PassRegs &r) {
+  const int64_t k0 = s + q0;
+  if (a.vec && q0 >= 0 && q0 + 8 <= len && k0 + 8 <= a.nnz) {
+    const U32x8 c = ld_stream_256(a.col_idx + k0);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) r.cv[j] = c.v[j];
+    if (VALS) {
+      const U32x8 v = ld_stream_256(a.val + k0);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) r.vv[j] = __uint_as_float(v.v[j]);
+    }
+  } else {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const bool in = (unsigned)(q0 + j) < (unsigned)len;
+      r.cv[j] = ld_stream_pred(a.col_idx + k0 + j, in);
+      r.vv[j] = VALS ? __uint_as_float(ld_stream_pred(a.val + k0 + j, in)) : 0.0f;
+    }
+  }
+}
+
+// The first pass of an item starts at p0 = -(s mod 8) for tiles (32-B aligned groups of 8);
+// a chunk is read lane-strided: pass = 256 consecutive entries, lane l takes entries
+// 8l .. 8l+7 of it, summed serially then across lanes — the same kernel path as tiles.
+__device__ __forceinline__ int first_p0(const WorkItem &it) { return -(int)(it.s & 7); }
+
+template <bool VALS, class Epi>
+__global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, GatherArgs a, Epi epi) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  float *xs = reinterpret_cast<float *>(smem_raw);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  WarpTileSmem &ws = reinterpret_cast<WarpTileSmem *>(smem_raw + (size_t)gp.n_hot * 4)[warp];
+  const int gw = blockIdx.x * kGatherWarps + warp, nwarps = gridDim.x * kGatherWarps;
+  if (lane == 0 && gw < gp.n_items) prefetch_item<VALS>(a, gp.items[gw]);
+  for (int i = threadIdx.x * 4; i < gp.n_hot; i += kGatherWarps * 32 * 4)
+    *reinterpret_cast<float4 *>(xs + i) = __ldg(reinterpret_cast<const float4 *>(gp.x_hot + i));
+  __syncthreads();
+  epi.init();
+  const uint64_t polx = policy_evict_last();
+  const unsigned lt = (1u << lane) - 1u;
+  if (gw >= gp.n_items) return;
+
+  // pipeline: `nx` holds the stream registers of the pass after the current one
+  WorkItem it = gp.items[gw];
+  WorkItem itn;  // the next item's descriptor (prefetched)
+  if (gw + nwarps < gp.n_items) itn = gp.items[gw + nwarps];
+  PassRegs nx;
+  load_pass<VALS>(a, it.s, (int)(it.e - it.s), first_p0(it) + 8 * lane, nx);
+  for (int idx = gw; idx < gp.n_items; idx += nwarps) {
+    const int64_t s = it.s;
+    const int len = (int)(it.e - s);
+    const bool has_next = idx + nwarps < gp.n_items;
+    if (lane == 0 && has_next) prefetch_item<VALS>(a, itn);
+    double dacc = 0.0;
+    int nnzr = 0;
+    if (it.j < 0) {  // tile: non-empty rows -> (offset, row) lists; empty rows finish here (y = 0)
+      const int nr = it.r1 - it.r0;
+      for (int rb = 0; rb < nr; rb += 32) {
+        const int r = rb + lane;
+        int off = 0, d = 0;
+        if (r < nr) {
+          const int64_t b = __ldg(a.row_ptr + it.r0 + r);
+          off = (int)(b - s);
+          d = (int)(__ldg(a.row_ptr + it.r0 + r + 1) - b);
+        }
+        const unsigned nz = __ballot_sync(0xffffffffu, r < nr && d > 0);
+        if (r < nr && d > 0) ws.nzrow[nnzr + __popc(nz & lt)] = (short)r;
+        if (r < nr && d == 0) dacc += epi(it.r0 + r, 0.0f);
+        nnzr += __popc(nz);
+        (void)off;
+      }
+    } else {  // a chunk is one row: its only start is offset 0
+      if (lane == 0) ws.nzrow[0] = 0;
+    }
+    __syncwarp();
+    int kcur = 0;        // number of row starts consumed so far in this item
+    int open_row = -1;   // local row open across the pass boundary
+    float carry = 0.0f;  // its partial sum
+    for (int p0 = first_p0(it);; p0 += 256) {  // >= 1 pass: it also hands the pipeline over
+      const int q0 = p0 + 8 * lane;
+      // (A) gathers of the current pass (its stream registers were loaded one pass ago)
+      float pr[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const bool in = (unsigned)(q0 + j) < (unsigned)len;
+        const float xv = gx((int32_t)nx.cv[j], in, xs, a.x, polx);
+        pr[j] = in ? (VALS ? nx.vv[j] * xv : xv) : 0.0f;
+      }
+      // issue the next pass's stream loads now (same item or the next item's first pass)
+      if (p0 + 256 < len) {
+        if (lane == 0 && p0 + 512 < len) prefetch_entries<VALS>(a, s + p0 + 512, s + min(len, p0 + 768));
+        load_pass<VALS>(a, s, len, q0 + 256, nx);
+      } else if (has_next) {
+        load_pass<VALS>(a, itn.s, (int)(itn.e - itn.s), first_p0(itn) + 8 * lane, nx);
+      }
+      // my 8 row-start flags (plan bit array; my segment is one 8-aligned byte of it)
+      unsigned fl = 0u;
+      {
+        const int64_t k0 = s + q0;  // 8-aligned
+        if (q0 + 8 > 0 && q0 < len) {
+          const uint32_t wv = __ldg(gp.rs_bits + (k0 >> 5));
+          fl = (wv >> (((int)(k0 >> 3) & 3) * 8)) & 0xffu;
+          const int lo = q0 < 0 ? -q0 : 0, hi = len - q0 < 8 ? len - q0 : 8;
+          fl &= (0xffu << lo) & (0xffu >> (8 - hi));  // entries of this item only
+          if (it.j >= 0 && q0 <= 0) fl |= 1u << lo;  // a chunk (re)starts its row at offset 0
+        }
+      }
+      // number of starts before my segment: exclusive scan of popc(fl)
+      int before = __popc(fl);
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, before, d);
+        if (lane >= d) before += t;
+      }
+      const int kpass = kcur;
+      kcur += __shfl_sync(0xffffffffu, before, 31);
+      before -= __popc(fl);
+      // THREAD-mapped rows: complete inside my segment -> emitted here
+      float head = 0.0f, cur = 0.0f;
+      int rank = before - 1;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        if (fl & (1u << j)) {
+          if (rank < before) head = cur;  // first start: what came before belongs to the open row
+          else dacc += epi(it.r0 + ws.nzrow[kpass + rank], cur);
+          ++rank;
+          cur = 0.0f;
+        }
+        cur += pr[j];
+      }
+      const bool F = fl != 0u;
+      if (!F) head = cur;
+      // WARP-mapped rows: segmented inclusive scan of (F ? tail : head) across lanes
+      float S = F ? cur : (lane == 0 ? head + carry : head);
+      bool G = F;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const float t = __shfl_up_sync(0xffffffffu, S, d);
+        const bool tg = __shfl_up_sync(0xffffffffu, G, d);
+        if (lane >= d) {
+          if (!G) S += t;
+          G = G || tg;
+        }
+      }
+      float E = __shfl_up_sync(0xffffffffu, S, 1);  // value entering my segment
+      if (lane == 0) E = carry;
+      if (F) {  // the row open at my segment start ends at my first flag
+        const int rr = before > 0 ? ws.nzrow[kpass + before - 1] : open_row;
+        if (rr >= 0) dacc += epi(it.r0 + rr, E + head);
+      }
+      const unsigned anyF = __ballot_sync(0xffffffffu, F);
+      carry = __shfl_sync(0xffffffffu, S, 31);
+      if (anyF) open_row = ws.nzrow[it.j < 0 ? kcur - 1 : 0];
+      __syncwarp();
+      if (p0 + 256 >= len) break;
+    }
+    // the row still open at the end of the item
+    if (lane == 0 && open_row >= 0) {
+      if (it.j < 0 || it.nch == 1) {
+        dacc += epi(it.r0 + open_row, carry);
+      } else {  // grid bin: partial of chunk c; the last chunk to finish combines in order
+        gp.partials[it.pbase + it.c] = carry;
+        cuda::atomic_ref<int, cuda::thread_scope_device> tk(gp.tickets[it.j]);
+        if (tk.fetch_add(1, cuda::memory_order_acq_rel) == it.nch - 1) {
+          double tot = 0.0;  // partials combined in chunk order, fp64 accumulator
+          for (int q = 0; q < it.nch; ++q) {
+            cuda::atomic_ref<float, cuda::thread_scope_device> pq(gp.partials[it.pbase + q]);
+            tot += (double)pq.load(cuda::memory_order_relaxed);
+          }
+          dacc += epi(it.r0, (float)tot);
+          tk.store(0, cuda::memory_order_relaxed);  // ready for the next call
+        }
+      }
+    }
+    if (Epi::kDangling) {
+      const double t = warp_sum_d(dacc);
+      if (lane == 0) gp.dpart[idx] = t;
+    }
+    __syncwarp();
+    if (has_next) {
+      it = itn;
+      if (idx + 2 * nwarps < gp.n_items) itn = gp.items[idx + 2 * nwarps];
+    }
+  }
+}
+
+// The paper's baseline (T1, P3@9322, P5@14490): one thread per row, serial inner
+// loop, no load balancing.  Used only as the in-build comparator.
+template <class Epi>
+__global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, GatherArgs a, Epi epi) {
+  epi.init();
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n_rows;
+       r += (int64_t)gridDim.x * blockDim.x) {
+    float acc = 0.0f;
+    for (int64_t k = a.row_ptr[r]; k < a.row_ptr[r + 1]; ++k)
+      acc += (a.val ? a.val[k] : 1.0f) * a.x[a.col_idx[k]];
+    epi(r, acc);
+  }
+}
+
+// x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu
+void build_xhot(inl_ctx ctx, inl_plan p, const float *x);
+
+template <bool VALS, class Epi>
+void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
+  const size_t smem = (size_t)gp.n_hot * 4 + (size_t)kGatherWarps * sizeof(WarpTileSmem);
+  auto kern = k_gather<VALS, Epi>;
+  static size_t configured = 0;  // per instantiation
+  if (smem > configured) {
+    INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    configured = smem;
+  }
+  int64_t grid = ctx->num_sms;
+  const int64_t need = (gp.n_items + kGatherWarps - 1) / kGatherWarps;
+  if (grid > need) grid = need;
+  kern<<<(int)grid, kGatherWarps * 32, smem, ctx->stream>>>(gp, a, epi);
+  INL_CUDA(cudaGetLastError());
+}
+
+// Host-side launcher for one full gather (tiles + long-row chunks) on a plan; x is the
+// dense vector (n_global) whose hot part is copied to the plan's x_hot first.
+template <bool VALS, class Epi>
+void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart) {
+  if (p->n_items == 0) return;
+  GatherArgs a = a_in;
+  a.col_idx = (const int32_t *)p->pcol.p;
+  GatherPlan gp;
+  gp.items = (const WorkItem *)p->items.p;
+  gp.n_items = (int)p->n_items;
+  gp.partials = (float *)p->partials.p;
+  gp.tickets = (int *)p->tickets.p;
+  gp.dpart = dpart;
+  gp.x_hot = (const float *)p->x_hot.p;
+  gp.n_hot = (int)((p->n_hot + 3) & ~3);
+  gp.rs_bits = (const uint32_t *)p->rs_bits.p;
+  build_xhot(ctx, p, a.x);
+  a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
+  launch_gather_t<VALS>(ctx, gp, a, epi);
+}
+
+}  // namespace inl

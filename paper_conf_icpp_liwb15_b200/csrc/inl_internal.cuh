@@ -1,0 +1,134 @@
+// inl_internal.cuh — shared internals of libinl.so (product path; no oracle code).
+#pragma once
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "inl.h"
+
+namespace inl {
+
+constexpr int kTileRows = 256;  // max rows per SpMV/PR warp tile
+
+// One unit of work of the fused gather kernel (one warp): a tile (j < 0: rows [r0, r1),
+// all of degree <= t_warp, nonzeros [s, e)) or one chunk c of long row r0 (j = long-row
+// index, nonzeros [s, e), nch chunks, partial slots from pbase).
+struct __align__(16) WorkItem {
+  int64_t s, e;
+  int32_t r0, r1, j, c, nch, pbase, pad0, pad1;
+};
+
+struct Status {
+  inl_status code = INL_OK;
+  std::string msg;
+};
+
+// Error carried from a failing CUDA/NCCL call up to the C-ABI boundary.
+struct Error {
+  inl_status code;
+  std::string msg;
+};
+
+[[noreturn]] void raise(inl_status code, const std::string &msg);
+
+#define INL_CUDA(call)                                                                     \
+  do {                                                                                     \
+    cudaError_t e_ = (call);                                                               \
+    if (e_ != cudaSuccess)                                                                 \
+      ::inl::raise(INL_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_) + " (" \
+                                     __FILE__ ":" + std::to_string(__LINE__) + ")");       \
+  } while (0)
+
+#define INL_NCCL(call)                                                                          \
+  do {                                                                                          \
+    ncclResult_t r_ = (call);                                                                   \
+    if (r_ != ncclSuccess)                                                                      \
+      ::inl::raise(INL_ERR_NCCL, std::string(#call) + ": " + ncclGetErrorString(r_) + " (" \
+                                     __FILE__ ":" + std::to_string(__LINE__) + ")");            \
+  } while (0)
+
+#define INL_CHECK(cond, msg)                                      \
+  do {                                                            \
+    if (!(cond)) ::inl::raise(INL_ERR_INVALID_ARGUMENT, (msg));   \
+  } while (0)
+
+// Growable device scratch buffer owned by a ctx or plan.
+struct DevBuf {
+  void *p = nullptr;
+  size_t bytes = 0;
+  void *get(size_t need);  // grows (cudaFree + cudaMalloc) when too small
+  void release();
+  ~DevBuf() { release(); }
+};
+
+struct Bins {
+  int t_thread, t_warp, t_block, grid_chunk, cta, flags;
+};
+Bins resolve_bins(const inl_bins *b);
+
+}  // namespace inl
+
+struct inl_ctx_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int num_sms = 148;
+  std::string last_error;
+  ncclComm_t comm = nullptr;
+  int nranks = 1, rank = 0;
+  // scratch
+  inl::DevBuf s_tmp, s_a, s_b, s_c, s_d, s_e, s_f, s_g;
+  inl::DevBuf h_rp, h_ci, h_val, h_x, h_y, h_w, h_od;  // host-staging device copies
+  int64_t *pinned = nullptr;                           // small pinned host scalars
+  int live_plans = 0;    // plans created on this ctx and not yet destroyed
+  bool closed = false;   // inl_ctx_destroy called; freed when the last plan goes
+};
+
+struct inl_plan_s {
+  inl_ctx ctx = nullptr;
+  // identity of the CSR it was built from
+  int64_t n_rows = 0, n_global = 0, row_begin = 0, nnz = 0;
+  const int64_t *row_ptr = nullptr;
+  const int32_t *col_idx = nullptr;
+  inl::Bins bins{};
+  // tiles: rows [tile_lo[t], tile_hi[t]) with every row of degree <= t_warp
+  int64_t n_tiles = 0;
+  inl::DevBuf tiles;  // int2 {lo, hi}
+  // long rows: degree > t_warp, cut into grid_chunk-sized chunks
+  int64_t n_long = 0, n_chunks = 0;
+  inl::DevBuf long_rows;    // int32 [n_long]
+  inl::DevBuf chunk_items;  // int2 {long index, chunk index} [n_chunks]
+  inl::DevBuf chunk_base;   // int32 [n_long] first chunk of each long row
+  inl::DevBuf partials;     // float [n_chunks]
+  inl::DevBuf tickets;      // int32 [n_long], zero between calls
+  inl::DevBuf dpart;        // double [n_items] (PageRank dangling partials, one per item)
+  // hot-column remap (plan-time): the n_hot most frequent columns are read from a
+  // shared-memory copy of x; pcol is col_idx with hot entries encoded 0x80000000 | h.
+  int64_t n_hot = 0;
+  inl::DevBuf hot_cols;     // int32 [n_hot] original column of hot slot h
+  inl::DevBuf pcol;         // int32 [nnz]
+  inl::DevBuf x_hot;        // float [n_hot] per-call copy of x[hot_cols]
+  inl::DevBuf rs_bits;      // uint32 [nnz/32 + 1]: bit k = entry k starts a non-empty row
+  int64_t n_items = 0;
+  inl::DevBuf items;        // WorkItem [n_items]: grid-bin chunks first, then tiles
+  inl_plan_info info{};
+};
+
+namespace inl {
+// plan.cu
+void build_plan(inl_plan p);
+// spmv.cu
+void spmv_run(inl_ctx ctx, inl_plan p, const float *val, const float *x, float *y);
+void spmv_thread_only(inl_ctx ctx, const inl_csr &A, const float *val, const float *x, float *y);
+// pagerank.cu
+void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damping, int iters,
+                  float *rank);
+// frontier.cu
+void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
+              uint32_t *dist, inl_stats *st);
+void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
+             inl_stats *st);
+// validate
+void csr_validate(inl_ctx ctx, const inl_csr &A);
+}  // namespace inl

@@ -1,0 +1,129 @@
+// pagerank.cu — PageRank pull iterations (PAPER.md P5@9262, P5@9781; reading R1)
+// on the binned gather.  One iteration = one fused gather launch (tiles + long
+// rows; epilogue computes PR', the next contribution and the dangling partials)
+// + one single-CTA fixed-order reduction of the dangling partials.  On P > 1
+// ranks the contribution slice and the rank's dangling sum are allgathered.
+#include "comm.h"
+#include "gather.cuh"
+
+namespace inl {
+
+namespace {
+
+// c[v] = PR^0(v) / outdeg(v) with PR^0 = 1/n; dangling count for D^0.
+__global__ void k_pr_init(const int32_t *__restrict__ od, int64_t n, float *__restrict__ c,
+                          unsigned long long *__restrict__ n_dangling) {
+  const float pr0 = (float)(1.0 / (double)n);
+  unsigned long long cnt = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    const int d = od[v];
+    c[v] = d > 0 ? pr0 / (float)d : 0.0f;
+    cnt += d == 0;
+  }
+  for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(n_dangling, cnt);
+}
+
+__global__ void k_pr_base0(const unsigned long long *__restrict__ n_dangling, int64_t n, double d,
+                           float *__restrict__ base) {
+  const double D = (double)*n_dangling * (1.0 / (double)n);  // sum of PR^0 over dangling pages
+  *base = (float)((1.0 - d) / (double)n + d * D / (double)n);
+}
+
+// Fixed-order sum of the dangling partials of this rank -> dloc.
+__global__ void __launch_bounds__(1024) k_pr_dsum(const double *__restrict__ dpart, int64_t m,
+                                                  double *__restrict__ dloc) {
+  __shared__ double red[32];
+  double s = 0.0;
+  for (int64_t i = threadIdx.x; i < m; i += 1024) s += dpart[i];
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int i = 0; i < 32; ++i) t += red[i];
+    *dloc = t;
+  }
+}
+
+// D = sum over ranks in rank order; base = (1-d)/n + d*D/n.
+__global__ void k_pr_base(const double *__restrict__ dall, int nranks, int64_t n, double d,
+                          float *__restrict__ base) {
+  double D = 0.0;
+  for (int r = 0; r < nranks; ++r) D += dall[r];
+  *base = (float)((1.0 - d) / (double)n + d * D / (double)n);
+}
+
+__global__ void k_fill(float *__restrict__ a, int64_t n, float v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    a[i] = v;
+}
+
+int grid_for(int64_t n, int sms) {
+  int64_t g = (n + 255) / 256;
+  if (g > (int64_t)sms * 16) g = (int64_t)sms * 16;
+  return g < 1 ? 1 : (int)g;
+}
+
+}  // namespace
+
+void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damping, int iters,
+                  float *rank) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = p->n_global;
+  if (n == 0) return;
+  if (iters == 0) {
+    k_fill<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(rank, n, (float)(1.0 / (double)n));
+    INL_CUDA(cudaGetLastError());
+    return;
+  }
+  const int P = ctx->nranks;
+  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  const int64_t B = DIST ? (n + P - 1) / P : n;  // allgather block (inl_partition_rows)
+  const int64_t npad = B * P;
+  float *c_cur = (float *)ctx->s_a.get(sizeof(float) * npad);
+  float *c_next = (float *)ctx->s_b.get(sizeof(float) * npad);
+  char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (P + 1));
+  float *base = (float *)scal;
+  unsigned long long *ndang = (unsigned long long *)(scal + 8);
+  double *dloc = (double *)(scal + 16);
+  double *dall = (double *)(scal + 256);
+  float *rank_pad = nullptr;
+  if (DIST) rank_pad = (float *)ctx->s_d.get(sizeof(float) * npad);
+
+  INL_CUDA(cudaMemsetAsync(ndang, 0, sizeof(unsigned long long), st));
+  k_pr_init<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(out_degree, n, c_cur, ndang);
+  k_pr_base0<<<1, 1, 0, st>>>(ndang, n, (double)damping, base);
+  INL_CUDA(cudaGetLastError());
+
+  const int64_t m = p->n_items;
+  double *dpart = (double *)p->dpart.p;
+  for (int t = 0; t < iters; ++t) {
+    const bool last = t + 1 == iters;
+    GatherArgs a{p->row_ptr, p->col_idx, nullptr, c_cur, p->nnz, p->n_rows,
+                 p->bins.t_thread, p->bins.t_warp, p->bins.t_block, p->bins.grid_chunk, false};
+    PrEpi epi{out_degree, c_next, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
+              p->row_begin, 0.0f};
+    launch_gather<false>(ctx, p, a, epi, dpart);
+    if (!last) {
+      k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
+      INL_CUDA(cudaGetLastError());
+      if (DIST) {
+        comm_allgather(ctx, c_next + (int64_t)ctx->rank * B, c_next, B, ncclFloat32, dloc, dall);
+      }
+      k_pr_base<<<1, 1, 0, st>>>(dall, P, n, (double)damping, base);
+      INL_CUDA(cudaGetLastError());
+      float *tmp = c_cur;
+      c_cur = c_next;
+      c_next = tmp;
+    }
+  }
+  if (DIST) {
+    comm_allgather(ctx, rank_pad + (int64_t)ctx->rank * B, rank_pad, B, ncclFloat32, nullptr, nullptr);
+    INL_CUDA(cudaMemcpyAsync(rank, rank_pad, sizeof(float) * n, cudaMemcpyDeviceToDevice, st));
+  }
+}
+
+}  // namespace inl

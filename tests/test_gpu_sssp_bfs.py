@@ -1,0 +1,116 @@
+"""GPU parity: inl_sssp / inl_bfs (CUDA through the C-ABI) vs oracle Dijkstra / queue BFS.
+
+Bar: bit-exact distances and levels (unique answers), every source; larger graphs
+add the exact O(m) certificate (tests/graphs.py) for every source."""
+import numpy as np
+import pytest
+import torch
+
+import inlgen
+import oracle
+from graphs import certify_bfs, certify_sssp, csr_from_edges
+from paper_conf_icpp_liwb15_b200 import inl
+
+pytestmark = pytest.mark.gpu
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    return inl.Ctx(0)
+
+
+@pytest.fixture(scope="module")
+def cfg1():
+    g = inlgen.host_build(12, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    w = inlgen.weights_host(g.row_ptr, g.col_idx)
+    return g, w
+
+
+def gpu_sssp(ctx, rp, ci, w, n, s, b=None):
+    A = inl.Csr(dev(rp), dev(ci), n)
+    d = torch.zeros(n, dtype=torch.int32, device="cuda")
+    plan = inl.Plan(ctx, A, b) if b is not None else None
+    st = inl.sssp(ctx, A, dev(w.view(np.int32)), s, d, plan)
+    return d.cpu().numpy().view(np.uint32), st
+
+
+def gpu_bfs(ctx, rp, ci, n, s, b=None):
+    A = inl.Csr(dev(rp), dev(ci), n)
+    lv = torch.zeros(n, dtype=torch.int32, device="cuda")
+    plan = inl.Plan(ctx, A, b) if b is not None else None
+    st = inl.bfs(ctx, A, s, lv, plan)
+    return lv.cpu().numpy(), st
+
+
+BINS = [None, dict(t_thread=-1, t_warp=32, t_block=128, grid_chunk=64),
+        dict(t_thread=1, t_warp=128, t_block=256, grid_chunk=64), dict(flags=inl.BINS_THREAD_ONLY),
+        dict(t_thread=64, t_warp=128, t_block=4096, grid_chunk=1000)]
+
+
+@pytest.mark.parametrize("bi", range(len(BINS)))
+def test_cfg1_all_sources_bit_exact(ctx, cfg1, bi):
+    g, w = cfg1
+    b = inl.bins(**BINS[bi]) if BINS[bi] is not None else None
+    for s in inlgen.sources(g.row_ptr, 8):
+        d, st = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, b)
+        assert np.array_equal(d, oracle.sssp(g.row_ptr, g.col_idx, w, s))
+        assert st["iterations"] >= 1
+        lv, st = gpu_bfs(ctx, g.row_ptr, g.col_idx, g.n_global, s, b)
+        assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col_idx, s))
+
+
+def test_small_graph_edge_cases(ctx):
+    rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3), (3, 1)], [5, 6, 7], symmetric=True)
+    d, _ = gpu_sssp(ctx, rp, ci, w, 6, 0)  # isolated source
+    assert d.tolist() == [0] + [0xFFFFFFFF] * 5
+    lv, _ = gpu_bfs(ctx, rp, ci, 6, 1)
+    assert lv.tolist() == [-1, 0, 1, 1, -1, -1]
+    rp = np.zeros(2, np.int64)
+    d, _ = gpu_sssp(ctx, rp, np.zeros(0, np.int32), np.zeros(0, np.uint32), 1, 0)
+    assert d.tolist() == [0]
+    # a star whose hub has degree far above every threshold (grid bin), path tail
+    n = 30000
+    e = [(0, i) for i in range(1, n - 100)] + [(i, i + 1) for i in range(n - 101, n - 1)]
+    rp, ci, w = csr_from_edges(n, e, np.arange(len(e)) % 255 + 1, symmetric=True)
+    for s in (0, n - 1, 5):
+        d, _ = gpu_sssp(ctx, rp, ci, w, n, s)
+        assert np.array_equal(d, oracle.sssp(rp, ci, w, s))
+        lv, _ = gpu_bfs(ctx, rp, ci, n, s)
+        assert np.array_equal(lv, oracle.bfs(rp, ci, s))
+
+
+def test_host_buffers(ctx, cfg1):
+    g, w = cfg1
+    s = inlgen.sources(g.row_ptr, 1)[0]
+    d = np.zeros(g.n_global, np.uint32)
+    inl.sssp(ctx, inl.Csr(g.row_ptr, g.col_idx, g.n_global), w, s, d)
+    assert np.array_equal(d, oracle.sssp(g.row_ptr, g.col_idx, w, s))
+    lv = np.zeros(g.n_global, np.int32)
+    inl.bfs(ctx, inl.Csr(g.row_ptr, g.col_idx, g.n_global), s, lv)
+    assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col_idx, s))
+
+
+def test_scale18_certificate_all_sources(ctx):
+    g = inlgen.dev_build(18, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    rp, ci = g["row_ptr"], g["col_idx"]
+    w = inlgen.weights_dev(rp, ci)
+    A = inl.Csr(rp, ci, g["n_global"])
+    plan = inl.Plan(ctx, A)
+    rph, cih, wh = rp.cpu().numpy(), ci.cpu().numpy(), w.cpu().numpy().view(np.uint32)
+    srcs = inlgen.sources(rph, 8)
+    for i, s in enumerate(srcs):
+        d = torch.zeros(g["n_global"], dtype=torch.int32, device="cuda")
+        inl.sssp(ctx, A, w, s, d, plan)
+        dh = d.cpu().numpy().view(np.uint32)
+        assert certify_sssp(rph, cih, wh, s, dh) is None
+        lv = torch.zeros(g["n_global"], dtype=torch.int32, device="cuda")
+        inl.bfs(ctx, A, s, lv, plan)
+        lvh = lv.cpu().numpy()
+        assert certify_bfs(rph, cih, s, lvh) is None
+        if i < 2:
+            assert np.array_equal(dh, oracle.sssp(rph, cih, wh, s))
+            assert np.array_equal(lvh, oracle.bfs(rph, cih, s))
