@@ -126,6 +126,25 @@ def partition_rows(n: int, nranks: int) -> list[int]:
     return [int(v) for v in b]
 
 
+def broadcast_unique_id(rank: int, group=None, device=None) -> np.ndarray:
+    """Rank 0 creates the NCCL unique id (inl_nccl_unique_id, no GPU needed) and every rank
+    receives it through torch.distributed; without a process group, returns rank 0's id."""
+    import torch
+    import torch.distributed as dist
+    uid = np.zeros(128, dtype=np.uint8)
+    if rank == 0:
+        rc = lib().inl_nccl_unique_id(uid.ctypes.data)
+        if rc != INL_OK:
+            raise InlError(rc, lib().inl_last_error(None).decode())
+    if dist.is_available() and dist.is_initialized():
+        t = torch.from_numpy(uid.copy())
+        if dist.get_backend(group) == "nccl":
+            t = t.cuda(device)
+        dist.broadcast(t, src=0, group=group)
+        uid = t.cpu().numpy().astype(np.uint8)
+    return uid
+
+
 class Ctx:
     """One library context per (process, device): stream, scratch, optional NCCL comm."""
 
@@ -144,17 +163,7 @@ class Ctx:
 
     def comm_init(self, nranks: int, rank: int, group=None) -> None:
         """NCCL communicator; the unique id travels through torch.distributed (gloo or nccl)."""
-        import torch
-        import torch.distributed as dist
-        uid = np.zeros(128, dtype=np.uint8)
-        if rank == 0:
-            _check(lib().inl_nccl_unique_id(uid.ctypes.data))
-        if nranks > 1 or dist.is_initialized():
-            t = torch.from_numpy(uid.copy())
-            if dist.get_backend(group) == "nccl":
-                t = t.cuda(self.device)
-            dist.broadcast(t, src=0, group=group)
-            uid = t.cpu().numpy().astype(np.uint8)
+        uid = broadcast_unique_id(rank, group, device=self.device)
         _check(lib().inl_comm_init(self.handle, uid.ctypes.data, nranks, rank), self)
         self.nranks, self.rank = nranks, rank
 
