@@ -55,7 +55,7 @@ struct WarpTileSmem {
 // hot slots that fit next to the per-warp tile scratch
 inline int64_t hot_capacity(int t_warp) {
   (void)t_warp;
-  int64_t b = kSmemBudget - (int64_t)kGatherWarps * (int64_t)sizeof(WarpTileSmem) - 1024;
+  int64_t b = kSmemBudget - (int64_t)kGatherWarps * (int64_t)sizeof(WarpTileSmem) - 2048;
   int64_t k = b / 4;
   if (k > kMaxHot) k = kMaxHot;
   return k < 0 ? 0 : (k & ~(int64_t)3);
@@ -117,17 +117,32 @@ struct GatherPlan {
   const uint32_t *rs_bits;  // [nnz/32 + 1] bit k set iff entry k starts a non-empty row
 };
 
-__device__ __forceinline__ float gather_x(int32_t c, const float *xs, const float *x, uint64_t polx) {
-  return c < 0 ? xs[c & 0x7fffffff] : ld_gather_f32(x + c, polx);
-}
 
-// x[c] for a remapped column: hot slots from shared memory, cold ones from global
-// (read-only path, L2 evict-last).  Branch-free.
-__device__ __forceinline__ float gx(int32_t c, bool in, const float *xs, const float *x, uint64_t polx) {
-  const bool hot = c < 0;
-  const float hv = xs[hot ? (c & 0x7fffffff) : 0];
-  const float cv = ld_gather_pred(x + (hot ? 0 : c), in && !hot, polx);
-  return hot ? hv : cv;
+// x[c] for a remapped column: hot slots (c = 0x80000000 | slot) from shared memory at
+// xs + (c << 2) (the shift drops the tag bit), cold columns from global memory
+// (read-only path).  One predicated load of each kind and a select: branch-free.
+__device__ __forceinline__ float gx(int32_t c, bool in, uint32_t xs_base, const float *x) {
+  float r;
+  asm("{\n\t"
+      ".reg .pred h, g, i;\n\t"
+      ".reg .b32 sa;\n\t"
+      ".reg .b64 ga;\n\t"
+      ".reg .f32 hv, cv;\n\t"
+      "setp.ne.b32 i, %2, 0;\n\t"
+      "setp.lt.and.s32 h, %1, 0, i;\n\t"
+      "setp.ge.and.s32 g, %1, 0, i;\n\t"
+      "shl.b32 sa, %1, 2;\n\t"
+      "add.u32 sa, sa, %3;\n\t"
+      "mov.f32 hv, 0f00000000;\n\t"
+      "mov.f32 cv, 0f00000000;\n\t"
+      "@h ld.shared.f32 hv, [sa];\n\t"
+      "mad.wide.s32 ga, %1, 4, %4;\n\t"
+      "@g ld.global.nc.f32 cv, [ga];\n\t"
+      "selp.f32 %0, hv, cv, h;\n\t"
+      "}"
+      : "=f"(r)
+      : "r"(c), "r"((int)in), "r"(xs_base), "l"(x));
+  return r;
 }
 
 __device__ __forceinline__ float lval(const float *val, int64_t k, bool in) {
@@ -156,8 +171,8 @@ struct PassRegs {
 
 template <bool VALS>
 __device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int len, int q0, PassRegs &r) {
-  const int64_t k0 = s + q0;
-  if (a.vec && q0 >= 0 && q0 + 8 <= len && k0 + 8 <= a.nnz) {
+  const int64_t k0 = s + q0;  // 8-aligned; the 32-B group lies inside the arrays unless at the end
+  if (a.vec && k0 + 8 <= a.nnz) {
     const U32x8 c = ld_stream_256(a.col_idx + k0);
 #pragma unroll
     for (int j = 0; j < 8; ++j) r.cv[j] = c.v[j];
@@ -186,14 +201,15 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float *xs = reinterpret_cast<float *>(smem_raw);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  WarpTileSmem &ws = reinterpret_cast<WarpTileSmem *>(smem_raw + (size_t)gp.n_hot * 4)[warp];
+  __shared__ WarpTileSmem ws_all[kGatherWarps];
+  WarpTileSmem &ws = ws_all[warp];
   const int gw = blockIdx.x * kGatherWarps + warp, nwarps = gridDim.x * kGatherWarps;
   if (lane == 0 && gw < gp.n_items) prefetch_item<VALS>(a, gp.items[gw]);
   for (int i = threadIdx.x * 4; i < gp.n_hot; i += kGatherWarps * 32 * 4)
     *reinterpret_cast<float4 *>(xs + i) = __ldg(reinterpret_cast<const float4 *>(gp.x_hot + i));
   __syncthreads();
   epi.init();
-  const uint64_t polx = policy_evict_last();
+  const uint32_t xs_base = smem_u32(xs);
   const unsigned lt = (1u << lane) - 1u;
   if (gw >= gp.n_items) return;
 
@@ -237,15 +253,22 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
       const int q0 = p0 + 8 * lane;
       // (A) gathers of the current pass (its stream registers were loaded one pass ago)
       float pr[8];
+      if (q0 >= 0 && q0 + 8 <= len) {  // whole group inside the item: no per-entry predicates
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const bool in = (unsigned)(q0 + j) < (unsigned)len;
-        const float xv = gx((int32_t)nx.cv[j], in, xs, a.x, polx);
-        pr[j] = in ? (VALS ? nx.vv[j] * xv : xv) : 0.0f;
+        for (int j = 0; j < 8; ++j) {
+          const float xv = gx((int32_t)nx.cv[j], true, xs_base, a.x);
+          pr[j] = VALS ? nx.vv[j] * xv : xv;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const bool in = (unsigned)(q0 + j) < (unsigned)len;
+          const float xv = gx((int32_t)nx.cv[j], in, xs_base, a.x);
+          pr[j] = in ? (VALS ? nx.vv[j] * xv : xv) : 0.0f;
+        }
       }
       // issue the next pass's stream loads now (same item or the next item's first pass)
       if (p0 + 256 < len) {
-        if (lane == 0 && p0 + 512 < len) prefetch_entries<VALS>(a, s + p0 + 512, s + min(len, p0 + 768));
         load_pass<VALS>(a, s, len, q0 + 256, nx);
       } else if (has_next) {
         load_pass<VALS>(a, itn.s, (int)(itn.e - itn.s), first_p0(itn) + 8 * lane, nx);
@@ -360,7 +383,7 @@ void build_xhot(inl_ctx ctx, inl_plan p, const float *x);
 
 template <bool VALS, class Epi>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
-  const size_t smem = (size_t)gp.n_hot * 4 + (size_t)kGatherWarps * sizeof(WarpTileSmem);
+  const size_t smem = (size_t)gp.n_hot * 4 + 16;  // xs[0] is read (then discarded) by cold gathers
   auto kern = k_gather<VALS, Epi>;
   static size_t configured = 0;  // per instantiation
   if (smem > configured) {
