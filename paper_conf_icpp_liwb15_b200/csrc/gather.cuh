@@ -115,6 +115,8 @@ struct GatherPlan {
   const float *x_hot;   // [n_hot]
   int n_hot;
   const uint32_t *rs_bits;  // [nnz/32 + 1] bit k set iff entry k starts a non-empty row
+  unsigned long long *ticket;  // work counter (monotone across launches)
+  unsigned long long base;     // its value at the start of this launch
 };
 
 
@@ -213,16 +215,26 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
   const unsigned lt = (1u << lane) - 1u;
   if (gw >= gp.n_items) return;
 
+  // dynamic schedule: a warp's first item is gw, later ones come from the work counter
+  // (items are ordered longest-first by the plan, so the tail is made of short tiles)
+  auto grab = [&]() -> int {
+    unsigned long long t = 0;
+    if (lane == 0) t = atomicAdd(gp.ticket, 1ull) - gp.base;
+    t = __shfl_sync(0xffffffffu, t, 0);
+    return (int)min(t + (unsigned long long)nwarps, (unsigned long long)gp.n_items);
+  };
   // pipeline: `nx` holds the stream registers of the pass after the current one
-  WorkItem it = gp.items[gw];
+  int idx = gw;
+  WorkItem it = gp.items[idx];
+  int nidx = grab();
   WorkItem itn;  // the next item's descriptor (prefetched)
-  if (gw + nwarps < gp.n_items) itn = gp.items[gw + nwarps];
+  if (nidx < gp.n_items) itn = gp.items[nidx];
   PassRegs nx;
   load_pass<VALS>(a, it.s, (int)(it.e - it.s), first_p0(it) + 8 * lane, nx);
-  for (int idx = gw; idx < gp.n_items; idx += nwarps) {
+  for (;;) {
     const int64_t s = it.s;
     const int len = (int)(it.e - s);
-    const bool has_next = idx + nwarps < gp.n_items;
+    const bool has_next = nidx < gp.n_items;
     if (lane == 0 && has_next) prefetch_item<VALS>(a, itn);
     double dacc = 0.0;
     int nnzr = 0;
@@ -357,10 +369,11 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
       if (lane == 0) gp.dpart[idx] = t;
     }
     __syncwarp();
-    if (has_next) {
-      it = itn;
-      if (idx + 2 * nwarps < gp.n_items) itn = gp.items[idx + 2 * nwarps];
-    }
+    if (!has_next) break;
+    idx = nidx;
+    it = itn;
+    nidx = grab();
+    if (nidx < gp.n_items) itn = gp.items[nidx];
   }
 }
 
@@ -413,6 +426,11 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
   gp.x_hot = (const float *)p->x_hot.p;
   gp.n_hot = (int)((p->n_hot + 3) & ~3);
   gp.rs_bits = (const uint32_t *)p->rs_bits.p;
+  gp.ticket = (unsigned long long *)p->ticket.p;
+  // each launch advances the counter by exactly n_items (successful grabs + one failing
+  // grab per active warp), so the next launch's base is known on the host: no reset
+  gp.base = p->ticket_base;
+  p->ticket_base += (unsigned long long)p->n_items;
   build_xhot(ctx, p, a.x);
   a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
   launch_gather_t<VALS>(ctx, gp, a, epi);

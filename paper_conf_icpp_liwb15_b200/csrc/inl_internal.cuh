@@ -110,6 +110,8 @@ struct inl_plan_s {
   inl::DevBuf pcol;         // int32 [nnz]
   inl::DevBuf x_hot;        // float [n_hot] per-call copy of x[hot_cols]
   inl::DevBuf rs_bits;      // uint32 [nnz/32 + 1]: bit k = entry k starts a non-empty row
+  inl::DevBuf ticket;       // uint64 dynamic-schedule counter of the gather kernel
+  unsigned long long ticket_base = 0;  // its value at the start of the next launch
   int64_t n_items = 0;
   inl::DevBuf items;        // WorkItem [n_items]: grid-bin chunks first, then tiles
   inl_plan_info info{};

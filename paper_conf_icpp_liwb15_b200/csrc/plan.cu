@@ -320,6 +320,8 @@ void build_plan(inl_plan p) {
     INL_CUDA(cudaGetLastError());
   }
   build_hot_remap(p);
+  INL_CUDA(cudaMemsetAsync(p->ticket.get(16), 0, 16, st));
+  p->ticket_base = 0;
   p->info.n_tiles = p->n_tiles;
   p->info.rows_thread = (int64_t)h_st[0];
   p->info.rows_warp = (int64_t)h_st[1];
