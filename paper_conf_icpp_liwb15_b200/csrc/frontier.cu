@@ -19,8 +19,11 @@
 //     trailing termination word.
 #include <cooperative_groups.h>
 
+#include <cub/block/block_scan.cuh>
+
 #include "comm.h"
 #include "inl_internal.cuh"
+#include "ptx.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -42,11 +45,12 @@ __device__ __forceinline__ void push(int32_t *q, int *cnt, int32_t v) {
 struct SsspOp {
   uint32_t *dist;       // [n_global (+1 flag word on P > 1)]
   const uint32_t *w;    // [nnz]
-  int *stamp;           // [n_global] (!DIST)
+  uint32_t *inq;        // !DIST: bitmap "already in the next frontier", cleared per iteration
   uint32_t *flag;       // P > 1: dist[n] cleared on any improvement
   int iter;
   int64_t row_begin;
   bool enqueue;         // !DIST: enqueue improved vertices directly
+  uint64_t pol_stream;  // L2 evict-first for the edge stream
   __device__ __forceinline__ uint32_t load(int32_t u) const {
     return *(volatile uint32_t *)(dist + row_begin + u);
   }
@@ -56,7 +60,8 @@ struct SsspOp {
       const uint32_t old = atomicMin(dist + v, nd);
       if (nd < old) {
         if (enqueue) {
-          if (atomicExch(stamp + v, iter) != iter) push(q, cnt, v);
+          const uint32_t bit = 1u << (v & 31);
+          if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, cnt, v);
         } else {
           *flag = 0u;
         }
@@ -72,6 +77,7 @@ struct BfsOp {
   int64_t n;
   int L;
   bool enqueue;      // !DIST
+  uint64_t pol_stream;
   __device__ __forceinline__ uint32_t load(int32_t) const { return 0u; }
   __device__ __forceinline__ void edge(uint32_t, int64_t, int32_t v, int32_t *q, int *cnt) const {
     const uint32_t bit = 1u << (v & 31);
@@ -105,6 +111,7 @@ struct ExpandArgs {
 
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
+  op.pol_stream = policy_evict_first();
   __shared__ int32_t lw[NT], lb[NT];
   __shared__ int nw, nb;
   __shared__ unsigned long long red[NW];
@@ -157,8 +164,106 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
   }
 }
 
+// Default expansion (dbuf-shared, P5@3623, B200 form): every frontier vertex of the
+// CTA's slice with degree <= t_warp is deferred to a shared-memory buffer of runs
+// (edge offset, degree prefix, dist); the CTA then runs the buffered inner loops over
+// their concatenation in windows of NT*kEdgesPerThread edges — thread t takes 8
+// consecutive edges of the window (one upper-bound search per window, then a walk),
+// so all threads do equal work and a warp touches consecutive edges.  Vertices of
+// larger degree go to the global grid buffer (dbuf-global) as grid_chunk pieces.
+constexpr int kEdgesPerThread = 8;
+
+template <class Op>
+__global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
+  op.pol_stream = policy_evict_first();
+  using Scan = cub::BlockScan<int, NT>;
+  __shared__ typename Scan::TempStorage scan_tmp;
+  __shared__ int64_t rs_s[NT];
+  __shared__ int off_s[NT + 1];
+  __shared__ uint32_t su_s[NT];
+  __shared__ unsigned long long red[NW];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int i = blockIdx.x * NT + tid;
+  int d = 0;
+  int64_t rs = 0;
+  uint32_t su = 0;
+  unsigned long long mydeg = 0;
+  if (i < a.nF) {
+    const int32_t u = a.F[i];
+    rs = a.rp[u];
+    const int64_t dd = a.rp[u + 1] - rs;
+    mydeg = (unsigned long long)dd;
+    su = op.load(u);
+    if (dd > a.t_warp) {  // grid bin: global delayed buffer
+      const int nch = (int)((dd + a.chunk - 1) / a.chunk);
+      const int base = atomicAdd(a.gcount, nch);
+      for (int c = 0; c < nch; ++c) a.gitems[base + c] = make_int2(u, c);
+    } else {
+      d = (int)dd;
+    }
+  }
+  // compact the non-empty runs (the buffer), then their edge offsets
+  int2 cnt_off = make_int2(d > 0 ? 1 : 0, d);
+  int2 excl, tot;
+  {
+    using Scan2 = cub::BlockScan<int2, NT>;
+    __shared__ typename Scan2::TempStorage scan2_tmp;
+    struct Add2 {
+      __device__ int2 operator()(int2 x, int2 y) const { return make_int2(x.x + y.x, x.y + y.y); }
+    };
+    Scan2(scan2_tmp).ExclusiveScan(cnt_off, excl, make_int2(0, 0), Add2(), tot);
+  }
+  (void)scan_tmp;
+  if (d > 0) {
+    rs_s[excl.x] = rs;
+    off_s[excl.x] = excl.y;
+    su_s[excl.x] = su;
+  }
+  const int nruns = tot.x, total = tot.y;
+  if (tid == 0) off_s[nruns] = total;
+  __syncthreads();
+  for (int w0 = 0; w0 < total; w0 += NT * kEdgesPerThread) {
+    int e = w0 + tid * kEdgesPerThread;
+    if (e >= total) continue;
+    int lo = 0, hi = nruns;  // last run with off_s[run] <= e
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (off_s[mid] <= e) lo = mid; else hi = mid;
+    }
+    int run = lo, rend = off_s[lo + 1];
+    int64_t kk[kEdgesPerThread];
+    uint32_t du[kEdgesPerThread];
+    int32_t vv[kEdgesPerThread];
+    bool in[kEdgesPerThread];
+#pragma unroll
+    for (int j = 0; j < kEdgesPerThread; ++j) {
+      in[j] = e + j < total;
+      if (in[j] && e + j >= rend) {  // runs are non-empty: one step reaches the next run
+        ++run;
+        rend = off_s[run + 1];
+      }
+      kk[j] = rs_s[run] + (e + j - off_s[run]);
+      du[j] = su_s[run];
+    }
+#pragma unroll
+    for (int j = 0; j < kEdgesPerThread; ++j) vv[j] = in[j] ? __ldg(a.col + kk[j]) : 0;
+#pragma unroll
+    for (int j = 0; j < kEdgesPerThread; ++j)
+      if (in[j]) op.edge(du[j], kk[j], vv[j], a.Fout, a.fcount);
+  }
+  for (int o = 16; o > 0; o >>= 1) mydeg += __shfl_xor_sync(0xffffffffu, mydeg, o);
+  if (lane == 0) red[warp] = mydeg;
+  __syncthreads();
+  if (tid == 0) {
+    unsigned long long s = 0;
+    for (int q = 0; q < NW; ++q) s += red[q];
+    if (s) atomicAdd(a.relaxed, s);
+  }
+}
+
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
+  op.pol_stream = policy_evict_first();
   const int n = *(volatile int *)a.gcount;
   for (int it = blockIdx.x; it < n; it += gridDim.x) {
     const int2 g = a.gitems[it];
@@ -167,7 +272,7 @@ __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
     const int64_t ke = min(ks + (int64_t)a.chunk, re);
     const uint32_t su = op.load(g.x);
     for (int64_t k = ks + threadIdx.x; k < ke; k += NT)
-      op.edge(su, k, __ldg(a.col + k), a.Fout, a.fcount);
+      op.edge(su, k, (int32_t)ld_stream_pol(a.col + k, op.pol_stream), a.Fout, a.fcount);
   }
 }
 
@@ -254,7 +359,12 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
   INL_CUDA(cudaMemsetAsync(f.counts, 0, 2 * sizeof(int), st));
   ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, b.grid_chunk,
                f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
-  if (nF > 0) k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
+  if (nF > 0) {
+    if (b.flags & INL_BINS_THREAD_ONLY)  // the paper's baseline: thread-mapped, no balancing
+      k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
+    else
+      k_expand_flat<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
+  }
   k_expand_grid<Op><<<ctx->num_sms * 2, NT, 0, st>>>(a, op);
   INL_CUDA(cudaGetLastError());
 }
@@ -286,13 +396,12 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
   uint32_t *D = dist;
   uint32_t *prev = nullptr;
-  int *stamp = nullptr;
+  uint32_t *inq = nullptr;
   if (DIST) {
     D = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * (n + 1));
     prev = (uint32_t *)ctx->s_e.get(sizeof(uint32_t) * (G.n_rows + 1));
   } else {
-    stamp = (int *)ctx->s_d.get(sizeof(int) * n);
-    INL_CUDA(cudaMemsetAsync(stamp, 0xFF, sizeof(int) * n, st));
+    inq = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * ((n + 31) / 32 + 1));
   }
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(D, n, source);
   INL_CUDA(cudaGetLastError());
@@ -310,7 +419,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
     ftotal += nF;
     if (!DIST) {
       if (nF == 0) break;
-      SsspOp op{D, w, stamp, nullptr, iters, 0, true};
+      INL_CUDA(cudaMemsetAsync(inq, 0, sizeof(uint32_t) * ((n + 31) / 32 + 1), st));
+      SsspOp op{D, w, inq, nullptr, iters, 0, true, 0};
       expand(ctx, G, b, f, nF, op);
       ++iters;
       nF = read_count(ctx, f.counts);
@@ -319,7 +429,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       // flag word D[n] = 1 ("no change"), cleared by any improvement on any rank
       const uint32_t one = 1u;
       INL_CUDA(cudaMemcpyAsync(D + n, &one, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
-      SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false};
+      SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false, 0};
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, D, n + 1, ncclUint32, ncclMin);
       ++iters;
@@ -361,14 +471,14 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
     ftotal += nF;
     if (!DIST) {
       if (nF == 0) break;
-      BfsOp op{bm, level, nullptr, n, L, true};
+      BfsOp op{bm, level, nullptr, n, L, true, 0};
       expand(ctx, G, b, f, nF, op);
       nF = read_count(ctx, f.counts);
       std::swap(f.F, f.Fout);
       ++L;
     } else {
       INL_CUDA(cudaMemsetAsync(next, 0, n + 1, st));
-      BfsOp op{bm, level, next, n, L, false};
+      BfsOp op{bm, level, next, n, L, false, 0};
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, next, n + 1, ncclUint8, ncclMax);
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, next + n, 1, cudaMemcpyDeviceToHost, st));

@@ -27,6 +27,13 @@ __device__ __forceinline__ uint32_t ld_stream_32(const void *p) {
   return r;
 }
 
+// Streaming 32-bit load with an L2 eviction policy (createpolicy), no L1 allocation.
+__device__ __forceinline__ uint32_t ld_stream_pol(const void *p, uint64_t pol) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+
 __device__ __forceinline__ uint64_t policy_evict_last() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
