@@ -165,27 +165,31 @@ __device__ __forceinline__ void prefetch_item(const GatherArgs &a, const WorkIte
   if (it.j < 0) prefetch_span(a.row_ptr + it.r0, a.row_ptr + it.r1 + 1, a.row_ptr + a.n_rows + 1);
 }
 
-// Stream registers of one pass: lane l holds entries q0 .. q0+7 of the item span.
+// Stream registers of one pass: lane l holds entries q0 .. q0+E-1 of the item span.
+template <int E>
 struct PassRegs {
-  uint32_t cv[8];
-  float vv[8];
+  uint32_t cv[E];
+  float vv[E];
 };
 
-template <bool VALS>
-__device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int len, int q0, PassRegs &r) {
-  const int64_t k0 = s + q0;  // 8-aligned; the 32-B group lies inside the arrays unless at the end
-  if (a.vec && k0 + 8 <= a.nnz) {
-    const U32x8 c = ld_stream_256(a.col_idx + k0);
+template <int E, bool VALS>
+__device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int len, int q0, PassRegs<E> &r) {
+  const int64_t k0 = s + q0;  // E-aligned; the group lies inside the arrays unless at the end
+  if (a.vec && k0 + E <= a.nnz) {
 #pragma unroll
-    for (int j = 0; j < 8; ++j) r.cv[j] = c.v[j];
-    if (VALS) {
-      const U32x8 v = ld_stream_256(a.val + k0);
+    for (int h = 0; h < E / 8; ++h) {
+      const U32x8 c = ld_stream_256(a.col_idx + k0 + 8 * h);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) r.vv[j] = __uint_as_float(v.v[j]);
+      for (int j = 0; j < 8; ++j) r.cv[8 * h + j] = c.v[j];
+      if (VALS) {
+        const U32x8 v = ld_stream_256(a.val + k0 + 8 * h);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) r.vv[8 * h + j] = __uint_as_float(v.v[j]);
+      }
     }
   } else {
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
+    for (int j = 0; j < E; ++j) {
       const bool in = (unsigned)(q0 + j) < (unsigned)len;
       r.cv[j] = ld_stream_pred(a.col_idx + k0 + j, in);
       r.vv[j] = VALS ? __uint_as_float(ld_stream_pred(a.val + k0 + j, in)) : 0.0f;
@@ -193,21 +197,25 @@ __device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int le
   }
 }
 
-// The first pass of an item starts at p0 = -(s mod 8) for tiles (32-B aligned groups of 8);
-// a chunk is read lane-strided: pass = 256 consecutive entries, lane l takes entries
-// 8l .. 8l+7 of it, summed serially then across lanes — the same kernel path as tiles.
-__device__ __forceinline__ int first_p0(const WorkItem &it) { return -(int)(it.s & 7); }
+// The first pass of an item starts at p0 = -(s mod E) (E-entry aligned groups); a pass
+// is 32*E consecutive entries, lane l takes entries E*l .. E*l+E-1 of it, summed serially
+// then across lanes — tiles and chunks take the same path.
+template <int E>
+__device__ __forceinline__ int first_p0(const WorkItem &it) { return -(int)(it.s & (E - 1)); }
 
-template <bool VALS, class Epi>
-__global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, GatherArgs a, Epi epi) {
+template <int E, bool VALS, class Epi>
+__global__ void __launch_bounds__(8192 / E, 1) k_gather(GatherPlan gp, GatherArgs a, Epi epi) {
+  constexpr int NWARP = 256 / E;  // 32 warps for E = 8, 16 for E = 16
+  constexpr int P = 32 * E;                     // entries per pass
+  constexpr unsigned EM = E == 32 ? 0xffffffffu : ((1u << E) - 1u);
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float *xs = reinterpret_cast<float *>(smem_raw);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  __shared__ WarpTileSmem ws_all[kGatherWarps];
+  __shared__ WarpTileSmem ws_all[NWARP];
   WarpTileSmem &ws = ws_all[warp];
-  const int gw = blockIdx.x * kGatherWarps + warp, nwarps = gridDim.x * kGatherWarps;
+  const int gw = blockIdx.x * NWARP + warp, nwarps = gridDim.x * NWARP;
   if (lane == 0 && gw < gp.n_items) prefetch_item<VALS>(a, gp.items[gw]);
-  for (int i = threadIdx.x * 4; i < gp.n_hot; i += kGatherWarps * 32 * 4)
+  for (int i = threadIdx.x * 4; i < gp.n_hot; i += NWARP * 32 * 4)
     *reinterpret_cast<float4 *>(xs + i) = __ldg(reinterpret_cast<const float4 *>(gp.x_hot + i));
   __syncthreads();
   epi.init();
@@ -229,8 +237,8 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
   int nidx = grab();
   WorkItem itn;  // the next item's descriptor (prefetched)
   if (nidx < gp.n_items) itn = gp.items[nidx];
-  PassRegs nx;
-  load_pass<VALS>(a, it.s, (int)(it.e - it.s), first_p0(it) + 8 * lane, nx);
+  PassRegs<E> nx;
+  load_pass<E, VALS>(a, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, nx);
   for (;;) {
     const int64_t s = it.s;
     const int len = (int)(it.e - s);
@@ -261,39 +269,39 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
     int kcur = 0;        // number of row starts consumed so far in this item
     int open_row = -1;   // local row open across the pass boundary
     float carry = 0.0f;  // its partial sum
-    for (int p0 = first_p0(it);; p0 += 256) {  // >= 1 pass: it also hands the pipeline over
-      const int q0 = p0 + 8 * lane;
+    for (int p0 = first_p0<E>(it);; p0 += P) {  // >= 1 pass: it also hands the pipeline over
+      const int q0 = p0 + E * lane;
       // (A) gathers of the current pass (its stream registers were loaded one pass ago)
-      float pr[8];
-      if (q0 >= 0 && q0 + 8 <= len) {  // whole group inside the item: no per-entry predicates
+      float pr[E];
+      if (q0 >= 0 && q0 + E <= len) {  // whole group inside the item: no per-entry predicates
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
+        for (int j = 0; j < E; ++j) {
           const float xv = gx((int32_t)nx.cv[j], true, xs_base, a.x);
           pr[j] = VALS ? nx.vv[j] * xv : xv;
         }
       } else {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
+        for (int j = 0; j < E; ++j) {
           const bool in = (unsigned)(q0 + j) < (unsigned)len;
           const float xv = gx((int32_t)nx.cv[j], in, xs_base, a.x);
           pr[j] = in ? (VALS ? nx.vv[j] * xv : xv) : 0.0f;
         }
       }
       // issue the next pass's stream loads now (same item or the next item's first pass)
-      if (p0 + 256 < len) {
-        load_pass<VALS>(a, s, len, q0 + 256, nx);
+      if (p0 + P < len) {
+        load_pass<E, VALS>(a, s, len, q0 + P, nx);
       } else if (has_next) {
-        load_pass<VALS>(a, itn.s, (int)(itn.e - itn.s), first_p0(itn) + 8 * lane, nx);
+        load_pass<E, VALS>(a, itn.s, (int)(itn.e - itn.s), first_p0<E>(itn) + E * lane, nx);
       }
-      // my 8 row-start flags (plan bit array; my segment is one 8-aligned byte of it)
+      // my E row-start flags (plan bit array; my segment is E-aligned within a 32-bit word)
       unsigned fl = 0u;
       {
-        const int64_t k0 = s + q0;  // 8-aligned
-        if (q0 + 8 > 0 && q0 < len) {
+        const int64_t k0 = s + q0;  // E-aligned
+        if (q0 + E > 0 && q0 < len) {
           const uint32_t wv = __ldg(gp.rs_bits + (k0 >> 5));
-          fl = (wv >> (((int)(k0 >> 3) & 3) * 8)) & 0xffu;
-          const int lo = q0 < 0 ? -q0 : 0, hi = len - q0 < 8 ? len - q0 : 8;
-          fl &= (0xffu << lo) & (0xffu >> (8 - hi));  // entries of this item only
+          fl = (wv >> ((int)(k0 & 31))) & EM;
+          const int lo = q0 < 0 ? -q0 : 0, hi = len - q0 < E ? len - q0 : E;
+          fl &= (EM << lo) & (EM >> (E - hi));  // entries of this item only
           if (it.j >= 0 && q0 <= 0) fl |= 1u << lo;  // a chunk (re)starts its row at offset 0
         }
       }
@@ -311,7 +319,7 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
       float head = 0.0f, cur = 0.0f;
       int rank = before - 1;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
+      for (int j = 0; j < E; ++j) {
         if (fl & (1u << j)) {
           if (rank < before) head = cur;  // first start: what came before belongs to the open row
           else dacc += epi(it.r0 + ws.nzrow[kpass + rank], cur);
@@ -334,17 +342,17 @@ __global__ void __launch_bounds__(kGatherWarps * 32, 1) k_gather(GatherPlan gp, 
           G = G || tg;
         }
       }
-      float E = __shfl_up_sync(0xffffffffu, S, 1);  // value entering my segment
-      if (lane == 0) E = carry;
+      float Ein = __shfl_up_sync(0xffffffffu, S, 1);  // value entering my segment
+      if (lane == 0) Ein = carry;
       if (F) {  // the row open at my segment start ends at my first flag
         const int rr = before > 0 ? ws.nzrow[kpass + before - 1] : open_row;
-        if (rr >= 0) dacc += epi(it.r0 + rr, E + head);
+        if (rr >= 0) dacc += epi(it.r0 + rr, Ein + head);
       }
       const unsigned anyF = __ballot_sync(0xffffffffu, F);
       carry = __shfl_sync(0xffffffffu, S, 31);
       if (anyF) open_row = ws.nzrow[it.j < 0 ? kcur - 1 : 0];
       __syncwarp();
-      if (p0 + 256 >= len) break;
+      if (p0 + P >= len) break;
     }
     // the row still open at the end of the item
     if (lane == 0 && open_row >= 0) {
@@ -394,20 +402,30 @@ __global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, Gath
 // x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu
 void build_xhot(inl_ctx ctx, inl_plan p, const float *x);
 
-template <bool VALS, class Epi>
+template <int E, bool VALS, class Epi>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
+  constexpr int NWARP = 256 / E;
   const size_t smem = (size_t)gp.n_hot * 4 + 16;  // xs[0] is read (then discarded) by cold gathers
-  auto kern = k_gather<VALS, Epi>;
+  auto kern = k_gather<E, VALS, Epi>;
   static size_t configured = 0;  // per instantiation
   if (smem > configured) {
     INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     configured = smem;
   }
   int64_t grid = ctx->num_sms;
-  const int64_t need = (gp.n_items + kGatherWarps - 1) / kGatherWarps;
+  const int64_t need = (gp.n_items + NWARP - 1) / NWARP;
   if (grid > need) grid = need;
-  kern<<<(int)grid, kGatherWarps * 32, smem, ctx->stream>>>(gp, a, epi);
+  kern<<<(int)grid, NWARP * 32, smem, ctx->stream>>>(gp, a, epi);
   INL_CUDA(cudaGetLastError());
+}
+
+inline int gather_entries_per_lane() {
+  static int e = 0;
+  if (!e) {  // 8 entries / lane with 32 warps measured best at scale 22 (16 / lane: 16 warps, slower)
+    e = 8;
+    if (const char *v = getenv("INL_GATHER_E")) e = atoi(v) == 16 ? 16 : 8;
+  }
+  return e;
 }
 
 // Host-side launcher for one full gather (tiles + long-row chunks) on a plan; x is the
@@ -433,7 +451,8 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
   p->ticket_base += (unsigned long long)p->n_items;
   build_xhot(ctx, p, a.x);
   a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
-  launch_gather_t<VALS>(ctx, gp, a, epi);
+  if (gather_entries_per_lane() == 8) launch_gather_t<8, VALS>(ctx, gp, a, epi);
+  else launch_gather_t<16, VALS>(ctx, gp, a, epi);
 }
 
 }  // namespace inl
