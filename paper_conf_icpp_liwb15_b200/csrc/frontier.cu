@@ -325,6 +325,61 @@ __global__ void k_bfs_apply(const uint8_t *__restrict__ next, int64_t n, int32_t
   }
 }
 
+// ---- direction-optimizing BFS (single GPU): bottom-up steps for large frontiers ----
+// One warp owns 32 consecutive vertices = one word of each bitmap, so no atomics: an
+// unvisited vertex scans its neighbours (thread-mapped, early exit at the first one in
+// the current frontier bitmap).
+__global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n,
+                                uint32_t *__restrict__ visited, const uint32_t *__restrict__ fcur,
+                                uint32_t *__restrict__ fnext, int32_t *__restrict__ level, int L,
+                                int *__restrict__ count) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nwords = (n + 31) / 32;
+  for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < nwords;
+       w += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t vis = visited[w];
+    const int64_t v = w * 32 + lane;
+    bool found = false;
+    if (v < n && !((vis >> lane) & 1u)) {
+      const int64_t e = rp[v + 1];
+      for (int64_t k = rp[v]; k < e; ++k) {
+        const int32_t u = __ldg(col + k);
+        if ((__ldg(fcur + (u >> 5)) >> (u & 31)) & 1u) {
+          found = true;
+          break;
+        }
+      }
+      if (found) level[v] = L + 1;
+    }
+    const uint32_t nw = __ballot_sync(0xffffffffu, found);
+    if (lane == 0) {
+      fnext[w] = nw;
+      if (nw) {
+        visited[w] = vis | nw;
+        atomicAdd(count, __popc(nw));
+      }
+    }
+  }
+}
+
+__global__ void k_queue_to_bitmap(const int32_t *__restrict__ q, int nq, uint32_t *__restrict__ bm) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nq; i += gridDim.x * blockDim.x)
+    atomicOr(bm + (q[i] >> 5), 1u << (q[i] & 31));
+}
+
+__global__ void k_bitmap_to_queue(const uint32_t *__restrict__ bm, int64_t n, int32_t *q, int *cnt) {
+  const int64_t nwords = (n + 31) / 32;
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nwords;
+       w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t b = bm[w];
+    while (b) {
+      const int t = __ffs(b) - 1;
+      b &= b - 1;
+      push(q, cnt, (int32_t)(w * 32 + t));
+    }
+  }
+}
+
 int grid_for(int64_t n, int sms) {
   int64_t g = (n + 255) / 256;
   if (g > (int64_t)sms * 16) g = (int64_t)sms * 16;
@@ -467,14 +522,47 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   }
   int L = 0;
   int64_t ftotal = 0;
+  // direction optimisation (Beamer et al.): bottom-up while the frontier holds more than
+  // n / kBuEnter vertices, top-down again once it falls below n / kBuLeave
+  const int64_t nwords = (n + 31) / 32;
+  uint32_t *fa = nullptr, *fb = nullptr;
+  bool bu = false;       // direction of the previous step
+  bool queue_ok = true;  // f.F holds the frontier (else the bitmap fa does)
+  const bool allow_bu = !(b.flags & INL_BINS_THREAD_ONLY) && n >= 4096;
+  if (allow_bu) {
+    fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
+    fb = fa + nwords + 1;
+  }
   for (;;) {
     ftotal += nF;
     if (!DIST) {
       if (nF == 0) break;
-      BfsOp op{bm, level, nullptr, n, L, true, 0};
-      expand(ctx, G, b, f, nF, op);
-      nF = read_count(ctx, f.counts);
-      std::swap(f.F, f.Fout);
+      const bool want_bu = allow_bu && (bu ? nF > n / 256 : nF > n / 24);
+      if (want_bu) {
+        if (queue_ok) {  // frontier queue -> bitmap
+          INL_CUDA(cudaMemsetAsync(fa, 0, sizeof(uint32_t) * nwords, st));
+          k_queue_to_bitmap<<<grid_for(nF, ctx->num_sms), 256, 0, st>>>(f.F, nF, fa);
+        }
+        INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+        k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
+                                                         f.counts);
+        INL_CUDA(cudaGetLastError());
+        nF = read_count(ctx, f.counts);
+        std::swap(fa, fb);
+        queue_ok = false;
+      } else {
+        if (!queue_ok) {  // bitmap -> frontier queue
+          INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+          k_bitmap_to_queue<<<grid_for(nwords, ctx->num_sms), 256, 0, st>>>(fa, n, f.F, f.counts);
+          INL_CUDA(cudaGetLastError());
+        }
+        BfsOp op{bm, level, nullptr, n, L, true, 0};
+        expand(ctx, G, b, f, nF, op);
+        nF = read_count(ctx, f.counts);
+        std::swap(f.F, f.Fout);
+        queue_ok = true;
+      }
+      bu = want_bu;
       ++L;
     } else {
       INL_CUDA(cudaMemsetAsync(next, 0, n + 1, st));
