@@ -18,6 +18,7 @@
 //     BFS allreduce-max of an n-byte next-frontier map, each with a
 //     trailing termination word.
 #include <cooperative_groups.h>
+#include <cstdlib>
 
 #include <cub/block/block_scan.cuh>
 
@@ -51,6 +52,10 @@ struct SsspOp {
   int64_t row_begin;
   bool enqueue;         // !DIST: enqueue improved vertices directly
   uint64_t pol_stream;  // L2 evict-first for the edge stream
+  uint32_t thr;         // near-far: vertices reaching dist >= thr go to the far pile
+  int32_t *far;         // far pile (each vertex at most once: `infar` bitmap)
+  int *far_count;
+  uint32_t *infar;
   __device__ __forceinline__ uint32_t load(int32_t u) const {
     return *(volatile uint32_t *)(dist + row_begin + u);
   }
@@ -60,8 +65,13 @@ struct SsspOp {
       const uint32_t old = atomicMin(dist + v, nd);
       if (nd < old) {
         if (enqueue) {
-          const uint32_t bit = 1u << (v & 31);
-          if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, cnt, v);
+          if (nd >= thr) {
+            const uint32_t bit = 1u << (v & 31);
+            if (!(atomicOr(infar + (v >> 5), bit) & bit)) push(far, far_count, v);
+          } else {
+            const uint32_t bit = 1u << (v & 31);
+            if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, cnt, v);
+          }
         } else {
           *flag = 0u;
         }
@@ -291,6 +301,24 @@ __global__ void k_init_bfs(int32_t *level, uint32_t *bm, int64_t n, int64_t s) {
   }
 }
 
+// Near-far: move far-pile vertices with lo <= dist < hi into the near frontier (once each);
+// keep those still >= hi (deduplicated through `keep`); drop the rest (already settled
+// in an earlier phase at a smaller distance).
+__global__ void k_far_split(const int32_t *__restrict__ far, int nfar, const uint32_t *__restrict__ dist,
+                            uint32_t lo, uint32_t hi, uint32_t *inq, uint32_t *keep, int32_t *q, int *qcnt,
+                            int32_t *far2, int *far2cnt) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nfar; i += gridDim.x * blockDim.x) {
+    const int32_t v = far[i];
+    const uint32_t d = dist[v];
+    const uint32_t bit = 1u << (v & 31);
+    if (d >= lo && d < hi) {
+      if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, qcnt, v);
+    } else if (d >= hi) {
+      if (!(atomicOr(keep + (v >> 5), bit) & bit)) push(far2, far2cnt, v);
+    }
+  }
+}
+
 // P > 1: vertices of the owned slice whose distance dropped -> next frontier.
 __global__ void k_sssp_collect(const uint32_t *__restrict__ dist, uint32_t *__restrict__ prev,
                                int64_t row_begin, int64_t n_rows, int32_t *q, int *cnt) {
@@ -386,6 +414,18 @@ int grid_for(int64_t n, int sms) {
   return g < 1 ? 1 : (int)g;
 }
 
+// Near-far bucket width (Davidson et al., IPDPS'14, "near-far" delta stepping); env
+// INL_SSSP_DELTA overrides (0xFFFFFFFF = plain frontier Bellman-Ford).
+uint32_t sssp_delta() {
+  static uint32_t d = 0;
+  if (!d) {
+    d = 32;  // measured best on R-MAT scale 23, w in [1, 255] (profiles/r01)
+    if (const char *e = getenv("INL_SSSP_DELTA")) d = (uint32_t)strtoul(e, nullptr, 10);
+    if (!d) d = 0xFFFFFFFFu;
+  }
+  return d;
+}
+
 struct FrontierBufs {
   int32_t *F, *Fout;
   int2 *gitems;
@@ -451,12 +491,26 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
   uint32_t *D = dist;
   uint32_t *prev = nullptr;
-  uint32_t *inq = nullptr;
+  uint32_t *inq = nullptr, *keep = nullptr;
+  const int64_t nwb = (n + 31) / 32 + 1;
+  int32_t *far_a = nullptr, *far_b = nullptr;
+  int *farcnt = nullptr;
+  int nfar = 0;
+  uint32_t delta = 0xFFFFFFFFu, thr = 0xFFFFFFFFu;
   if (DIST) {
     D = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * (n + 1));
     prev = (uint32_t *)ctx->s_e.get(sizeof(uint32_t) * (G.n_rows + 1));
   } else {
-    inq = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * ((n + 31) / 32 + 1));
+    inq = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 2 * nwb);
+    keep = inq + nwb;
+    // far piles hold each vertex at most once (`keep` doubles as the in-far bitmap)
+    far_a = (int32_t *)ctx->s_g.get(sizeof(int32_t) * (2 * n + 16));
+    far_b = far_a + n + 8;
+    farcnt = (int *)ctx->s_e.get(16);
+    INL_CUDA(cudaMemsetAsync(farcnt, 0, 16, st));
+    INL_CUDA(cudaMemsetAsync(keep, 0, sizeof(uint32_t) * nwb, st));
+    delta = b.flags & INL_BINS_THREAD_ONLY ? 0xFFFFFFFFu : sssp_delta();
+    thr = delta;
   }
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(D, n, source);
   INL_CUDA(cudaGetLastError());
@@ -473,18 +527,41 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   for (;;) {
     ftotal += nF;
     if (!DIST) {
-      if (nF == 0) break;
-      INL_CUDA(cudaMemsetAsync(inq, 0, sizeof(uint32_t) * ((n + 31) / 32 + 1), st));
-      SsspOp op{D, w, inq, nullptr, iters, 0, true, 0};
+      if (nF == 0) {  // near frontier exhausted: advance the threshold, pull in the far pile
+        if (nfar == 0) break;
+        const uint32_t lo = thr;
+        thr = thr > 0xFFFFFFFFu - delta ? 0xFFFFFFFFu : thr + delta;
+        INL_CUDA(cudaMemsetAsync(inq, 0, sizeof(uint32_t) * nwb, st));
+        INL_CUDA(cudaMemsetAsync(keep, 0, sizeof(uint32_t) * nwb, st));
+        INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+        INL_CUDA(cudaMemsetAsync(farcnt + 1, 0, sizeof(int), st));
+        k_far_split<<<grid_for(nfar, ctx->num_sms), 256, 0, st>>>(far_a, nfar, D, lo, thr, inq, keep, f.F,
+                                                                 f.counts, far_b, farcnt + 1);
+        INL_CUDA(cudaGetLastError());
+        INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, sizeof(int), cudaMemcpyDeviceToHost, st));
+        INL_CUDA(cudaMemcpyAsync((int *)ctx->pinned + 1, farcnt + 1, sizeof(int), cudaMemcpyDeviceToHost, st));
+        INL_CUDA(cudaStreamSynchronize(st));
+        nF = ((volatile int *)ctx->pinned)[0];
+        nfar = ((volatile int *)ctx->pinned)[1];
+        std::swap(far_a, far_b);
+        INL_CUDA(cudaMemcpyAsync(farcnt, farcnt + 1, sizeof(int), cudaMemcpyDeviceToDevice, st));
+        continue;
+      }
+      INL_CUDA(cudaMemsetAsync(inq, 0, sizeof(uint32_t) * nwb, st));
+      SsspOp op{D, w, inq, nullptr, iters, 0, true, 0, thr, far_a, farcnt, keep};
       expand(ctx, G, b, f, nF, op);
       ++iters;
-      nF = read_count(ctx, f.counts);
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, sizeof(int), cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaMemcpyAsync((int *)ctx->pinned + 1, farcnt, sizeof(int), cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaStreamSynchronize(st));
+      nF = ((volatile int *)ctx->pinned)[0];
+      nfar = ((volatile int *)ctx->pinned)[1];
       std::swap(f.F, f.Fout);
     } else {
       // flag word D[n] = 1 ("no change"), cleared by any improvement on any rank
       const uint32_t one = 1u;
       INL_CUDA(cudaMemcpyAsync(D + n, &one, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
-      SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false, 0};
+      SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false, 0, 0xFFFFFFFFu, nullptr, nullptr, nullptr};
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, D, n + 1, ncclUint32, ncclMin);
       ++iters;
