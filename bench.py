@@ -201,13 +201,13 @@ def run_inl(a):
         step = lambda: inl.spmv(ctx, A, W["val"], W["x"], y, plan)  # noqa: E731
         units_local = nnz_local
         bytes_local = spmv_bytes(nnz_local, A.n_rows, A.n_global)
-        launches_per_step = 1
+        launches_per_step = 2 if info["bins"]["flags"] == 0 else 1  # k_build_xhot + k_gather
     elif a.op == "pagerank":
         r = torch.empty(A.n_global, device="cuda")
         step = lambda: inl.pagerank(ctx, A, g["out_degree"], r, 0.85, a.iterations, plan)  # noqa: E731
         units_local = nnz_local * a.iterations
         bytes_local = pagerank_bytes_per_iter(nnz_local, A.n_rows, A.n_global) * a.iterations
-        launches_per_step = 3 + 3 * a.iterations
+        launches_per_step = 3 + 4 * a.iterations  # init; per iteration xhot + gather + dsum + base
     else:
         srcs = inlgen.sources(g["row_ptr"].cpu().numpy(), 8) if world == 1 else [0]
         if world > 1:
@@ -303,7 +303,7 @@ def run_inl(a):
         out["roofline"] = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak, "unit": "GB/s",
                            "frac": round(frac, 4), "peak_source": peak_src,
                            "frac_of_8TBs": round(achieved_gbs / 8000.0, 4),
-                           "kernel": "k_gather (fused tile + grid-bin gather)" if a.op in ("spmv", "pagerank") else "k_expand",
+                           "kernel": "k_gather (fused tile + grid-bin gather)" if a.op in ("spmv", "pagerank") else "k_expand_flat",
                            "alg_bytes_per_step_per_gpu": int(bytes_total / world / a.steps),
                            "traffic": traffic_lookup(a.op, scale)}
         out["plan"] = info

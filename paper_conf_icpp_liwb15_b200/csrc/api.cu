@@ -158,9 +158,12 @@ inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user, inl_plan *transi
     INL_CHECK(same_csr(user, A), "plan was created for a different CSR (pointers or sizes differ)");
     return user;
   }
-  inl_plan p = new inl_plan_s();
-  *transient_holder = p;
+  // the ctx keeps one transient plan whose buffers are reused across calls
+  if (!ctx->tplan) ctx->tplan = new inl_plan_s();
+  inl_plan p = ctx->tplan;
+  (void)transient_holder;
   p->ctx = ctx;
+  p->transient = true;
   p->n_rows = A.n_rows;
   p->n_global = A.n_global;
   p->row_begin = A.row_begin;
@@ -172,9 +175,8 @@ inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user, inl_plan *transi
   return p;
 }
 
-struct PlanHolder {
+struct PlanHolder {  // transient plans now live in the ctx (ctx->tplan); kept for clarity
   inl_plan p = nullptr;
-  ~PlanHolder() { delete p; }
 };
 
 inl_status fail(inl_ctx ctx, inl_status code, const std::string &msg) {
@@ -306,6 +308,7 @@ static void free_ctx(inl_ctx ctx) {
   cudaStreamSynchronize(ctx->stream);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
+  delete ctx->tplan;
   delete ctx;  // DevBuf destructors free device scratch
   if (old >= 0) cudaSetDevice(old);
 }

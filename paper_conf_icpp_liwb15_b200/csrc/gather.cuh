@@ -434,7 +434,7 @@ template <bool VALS, class Epi>
 void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart) {
   if (p->n_items == 0) return;
   GatherArgs a = a_in;
-  a.col_idx = (const int32_t *)p->pcol.p;
+  if (p->n_hot > 0) a.col_idx = (const int32_t *)p->pcol.p;  // hot columns remapped
   GatherPlan gp;
   gp.items = (const WorkItem *)p->items.p;
   gp.n_items = (int)p->n_items;

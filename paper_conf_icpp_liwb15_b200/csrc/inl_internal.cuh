@@ -82,6 +82,7 @@ struct inl_ctx_s {
   inl::DevBuf h_rp, h_ci, h_val, h_x, h_y, h_w, h_od;  // host-staging device copies
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
+  struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
   bool closed = false;   // inl_ctx_destroy called; freed when the last plan goes
 };
 
@@ -115,6 +116,7 @@ struct inl_plan_s {
   int64_t n_items = 0;
   inl::DevBuf items;        // WorkItem [n_items]: grid-bin chunks first, then tiles
   inl_plan_info info{};
+  bool transient = false;  // built inside a call: no hot-column remap (pcol unused)
 };
 
 namespace inl {

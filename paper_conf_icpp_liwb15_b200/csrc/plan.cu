@@ -188,14 +188,12 @@ void build_hot_remap(inl_plan p) {
   const int64_t ng = p->n_global, nnz = p->nnz;
   int64_t n_hot = hot_capacity(p->bins.t_warp);
   if (const char *e = getenv("INL_HOT_K")) n_hot = atoll(e) & ~(int64_t)3;
+  if (p->transient) n_hot = 0;  // a one-shot call does not amortise the remap
   if (n_hot > ng) n_hot = ng;
   if (nnz == 0) n_hot = 0;
-  int32_t *pcol = (int32_t *)p->pcol.get(sizeof(int32_t) * (nnz > 0 ? nnz : 1));
   p->n_hot = n_hot;
-  if (n_hot == 0) {
-    if (nnz) INL_CUDA(cudaMemcpyAsync(pcol, p->col_idx, sizeof(int32_t) * nnz, cudaMemcpyDeviceToDevice, st));
-    return;
-  }
+  if (n_hot == 0) return;  // the gather reads col_idx directly
+  int32_t *pcol = (int32_t *)p->pcol.get(sizeof(int32_t) * (nnz > 0 ? nnz : 1));
   int32_t *cnt = (int32_t *)ctx->s_a.get(sizeof(int32_t) * ng);
   int32_t *cnt_sorted = (int32_t *)ctx->s_b.get(sizeof(int32_t) * ng);
   int32_t *ids = (int32_t *)ctx->s_c.get(sizeof(int32_t) * ng);
