@@ -203,9 +203,9 @@ __device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int le
 template <int E>
 __device__ __forceinline__ int first_p0(const WorkItem &it) { return -(int)(it.s & (E - 1)); }
 
-template <int E, bool VALS, class Epi>
-__global__ void __launch_bounds__(8192 / E, 1) k_gather(GatherPlan gp, GatherArgs a, Epi epi) {
-  constexpr int NWARP = 256 / E;  // 32 warps for E = 8, 16 for E = 16
+template <int E, bool VALS, class Epi, int NWARP = 256 / E>
+__global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherArgs a, Epi epi) {
+  // NWARP: 32 warps for E = 8 (64 registers), 24 (85 registers) or 16 for E = 16
   constexpr int P = 32 * E;                     // entries per pass
   constexpr unsigned EM = E == 32 ? 0xffffffffu : ((1u << E) - 1u);
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -402,11 +402,10 @@ __global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, Gath
 // x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu
 void build_xhot(inl_ctx ctx, inl_plan p, const float *x);
 
-template <int E, bool VALS, class Epi>
+template <int E, bool VALS, class Epi, int NWARP = 256 / E>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
-  constexpr int NWARP = 256 / E;
   const size_t smem = (size_t)gp.n_hot * 4 + 16;  // xs[0] is read (then discarded) by cold gathers
-  auto kern = k_gather<E, VALS, Epi>;
+  auto kern = k_gather<E, VALS, Epi, NWARP>;
   static size_t configured = 0;  // per instantiation
   if (smem > configured) {
     INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -451,8 +450,11 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
   p->ticket_base += (unsigned long long)p->n_items;
   build_xhot(ctx, p, a.x);
   a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
-  if (gather_entries_per_lane() == 8) launch_gather_t<8, VALS>(ctx, gp, a, epi);
-  else launch_gather_t<16, VALS>(ctx, gp, a, epi);
+  static int w24 = -1;
+  if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;
+  if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi);
+  else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi);
+  else launch_gather_t<8, VALS>(ctx, gp, a, epi);
 }
 
 }  // namespace inl
