@@ -271,6 +271,8 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
   }
 }
 
+// Grid bin (dbuf-global, P5@2721): pieces of grid_chunk edges of the large-degree
+// frontier vertices, one CTA per piece (grid-stride); each thread keeps 8 edges in flight.
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
@@ -281,8 +283,19 @@ __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
     const int64_t ks = rs + (int64_t)g.y * a.chunk;
     const int64_t ke = min(ks + (int64_t)a.chunk, re);
     const uint32_t su = op.load(g.x);
-    for (int64_t k = ks + threadIdx.x; k < ke; k += NT)
-      op.edge(su, k, (int32_t)ld_stream_pol(a.col + k, op.pol_stream), a.Fout, a.fcount);
+    for (int64_t k0 = ks + threadIdx.x; k0 < ke; k0 += NT * kEdgesPerThread) {
+      int32_t vv[kEdgesPerThread];
+#pragma unroll
+      for (int j = 0; j < kEdgesPerThread; ++j) {
+        const int64_t k = k0 + (int64_t)j * NT;
+        vv[j] = k < ke ? (int32_t)ld_stream_pol(a.col + k, op.pol_stream) : 0;
+      }
+#pragma unroll
+      for (int j = 0; j < kEdgesPerThread; ++j) {
+        const int64_t k = k0 + (int64_t)j * NT;
+        if (k < ke) op.edge(su, k, vv[j], a.Fout, a.fcount);
+      }
+    }
   }
 }
 
@@ -452,7 +465,7 @@ template <class Op>
 void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int nF, const Op &op) {
   cudaStream_t st = ctx->stream;
   INL_CUDA(cudaMemsetAsync(f.counts, 0, 2 * sizeof(int), st));
-  ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, b.grid_chunk,
+  ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
                f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
   if (nF > 0) {
     if (b.flags & INL_BINS_THREAD_ONLY)  // the paper's baseline: thread-mapped, no balancing
@@ -460,7 +473,7 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
     else
       k_expand_flat<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
   }
-  k_expand_grid<Op><<<ctx->num_sms * 2, NT, 0, st>>>(a, op);
+  k_expand_grid<Op><<<ctx->num_sms * 8, NT, 0, st>>>(a, op);
   INL_CUDA(cudaGetLastError());
 }
 
