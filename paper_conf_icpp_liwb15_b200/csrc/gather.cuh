@@ -147,6 +147,29 @@ __device__ __forceinline__ float gx(int32_t c, bool in, uint32_t xs_base, const 
   return r;
 }
 
+// gx for an entry known to be inside the item (no `in` predicate).
+__device__ __forceinline__ float gx_in(int32_t c, uint32_t xs_base, const float *x) {
+  float r;
+  asm("{\n\t"
+      ".reg .pred h;\n\t"
+      ".reg .b32 sa;\n\t"
+      ".reg .b64 ga;\n\t"
+      ".reg .f32 hv, cv;\n\t"
+      "setp.lt.s32 h, %1, 0;\n\t"
+      "shl.b32 sa, %1, 2;\n\t"
+      "add.u32 sa, sa, %2;\n\t"
+      "mov.f32 hv, 0f00000000;\n\t"
+      "mov.f32 cv, 0f00000000;\n\t"
+      "@h ld.shared.f32 hv, [sa];\n\t"
+      "mad.wide.s32 ga, %1, 4, %3;\n\t"
+      "@!h ld.global.nc.f32 cv, [ga];\n\t"
+      "selp.f32 %0, hv, cv, h;\n\t"
+      "}"
+      : "=f"(r)
+      : "r"(c), "r"(xs_base), "l"(x));
+  return r;
+}
+
 __device__ __forceinline__ float lval(const float *val, int64_t k, bool in) {
   return val ? __uint_as_float(ld_stream_pred(val + k, in)) : (in ? 1.0f : 0.0f);
 }
@@ -276,7 +299,7 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
       if (q0 >= 0 && q0 + E <= len) {  // whole group inside the item: no per-entry predicates
 #pragma unroll
         for (int j = 0; j < E; ++j) {
-          const float xv = gx((int32_t)nx.cv[j], true, xs_base, a.x);
+          const float xv = gx_in((int32_t)nx.cv[j], xs_base, a.x);
           pr[j] = VALS ? nx.vv[j] * xv : xv;
         }
       } else {
