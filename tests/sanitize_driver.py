@@ -1,0 +1,43 @@
+"""Small end-to-end run of every op through the C-ABI (used under compute-sanitizer)."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import inlgen  # noqa: E402
+from paper_conf_icpp_liwb15_b200 import inl  # noqa: E402
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def main():
+    ctx = inl.Ctx(0)
+    g = inlgen.host_build(10, 16, seed=1)
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    y = torch.empty(A.n_rows, device="cuda")
+    for b in (None, inl.bins(t_thread=2, t_warp=32, t_block=64, grid_chunk=48)):
+        inl.spmv(ctx, A, dev(inlgen.values_host(g.row_ptr, g.col_idx)), dev(inlgen.vector_host(g.n_global)), y,
+                 inl.Plan(ctx, A, b))
+    inl.spmv(ctx, A, dev(inlgen.values_host(g.row_ptr, g.col_idx)), dev(inlgen.vector_host(g.n_global)), y)
+    t = inlgen.host_build(10, 16, seed=1, flags=inlgen.TRANSPOSE)
+    At = inl.Csr(dev(t.row_ptr), dev(t.col_idx), t.n_global)
+    r = torch.empty(t.n_global, device="cuda")
+    inl.pagerank(ctx, At, dev(t.out_degree), r, 0.85, 5, inl.Plan(ctx, At))
+    s = inlgen.host_build(12, 16, seed=1, flags=inlgen.SYMMETRIC)
+    As = inl.Csr(dev(s.row_ptr), dev(s.col_idx), s.n_global)
+    w = dev(inlgen.weights_host(s.row_ptr, s.col_idx).view(np.int32))
+    d = torch.empty(s.n_global, dtype=torch.int32, device="cuda")
+    src = inlgen.sources(s.row_ptr, 1)[0]
+    inl.sssp(ctx, As, w, src, d)
+    inl.bfs(ctx, As, src, d)
+    torch.cuda.synchronize()
+    print("sanitize driver ok")
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,24 @@
+"""compute-sanitizer (memcheck, racecheck, synccheck) over every kernel of the path on small
+inputs (SURVEY §4.3 tests/sanitize): no out-of-bounds access, no shared-memory race."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer(tool):
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    cmd = [cs, "--tool", tool, "--error-exitcode", "17", "--print-limit", "20"]
+    if tool == "memcheck":
+        cmd += ["--leak-check", "no"]
+    cmd += [sys.executable, os.path.join(HERE, "sanitize_driver.py")]
+    p = subprocess.run(cmd, capture_output=True, text=True, timeout=900)
+    out = p.stdout + p.stderr
+    assert p.returncode == 0, out[-4000:]
+    assert "sanitize driver ok" in out
