@@ -78,7 +78,8 @@ struct SpmvEpi {
 // dangling pages so the warp can form its fixed-order partial of D'.
 struct PrEpi {
   const int32_t *out_degree;  // [n_global]
-  float *c_next;              // [n_global]; this rank writes its own rows
+  float *c_next;              // compacted contributions; this rank writes its own rows
+  const int32_t *cidx;        // [n_global] compact (exchange-space) index of v, -1 if dangling
   float *rank_out;            // [n_global] or nullptr
   const float *base_ptr;      // device scalar
   float damping;
@@ -90,7 +91,7 @@ struct PrEpi {
     const int64_t v = row_begin + r;
     const float pr = fmaf(damping, s, base);
     const int od = __ldg(out_degree + v);
-    c_next[v] = od > 0 ? pr / (float)od : 0.0f;
+    if (od > 0) c_next[__ldg(cidx + v)] = pr / (float)od;
     if (rank_out) rank_out[v] = pr;
     return od == 0 ? (double)pr : 0.0;
   }
@@ -422,8 +423,9 @@ __global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, Gath
   }
 }
 
-// x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu
-void build_xhot(inl_ctx ctx, inl_plan p, const float *x);
+// x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu.
+// hot_cols: NULL = the plan's list, else a list in another column space.
+void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols = nullptr);
 
 template <int E, bool VALS, class Epi, int NWARP = 256 / E>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
@@ -452,11 +454,14 @@ inline int gather_entries_per_lane() {
 
 // Host-side launcher for one full gather (tiles + long-row chunks) on a plan; x is the
 // dense vector (n_global) whose hot part is copied to the plan's x_hot first.
+// col_over / hot_over: a column space other than the plan's (PageRank's compacted one).
 template <bool VALS, class Epi>
-void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart) {
+void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart,
+                   const int32_t *col_over = nullptr, const int32_t *hot_over = nullptr) {
   if (p->n_items == 0) return;
   GatherArgs a = a_in;
-  if (p->n_hot > 0) a.col_idx = (const int32_t *)p->pcol.p;  // hot columns remapped
+  if (col_over) a.col_idx = col_over;
+  else if (p->n_hot > 0) a.col_idx = (const int32_t *)p->pcol.p;  // hot columns remapped
   GatherPlan gp;
   gp.items = (const WorkItem *)p->items.p;
   gp.n_items = (int)p->n_items;
@@ -471,7 +476,7 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
   // grab per active warp), so the next launch's base is known on the host: no reset
   gp.base = p->ticket_base;
   p->ticket_base += (unsigned long long)p->n_items;
-  build_xhot(ctx, p, a.x);
+  build_xhot(ctx, p, a.x, hot_over);
   a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
   static int w24 = -1;
   if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;

@@ -117,6 +117,13 @@ struct inl_plan_s {
   inl::DevBuf items;        // WorkItem [n_items]: grid-bin chunks first, then tiles
   inl_plan_info info{};
   bool transient = false;  // built inside a call: no hot-column remap (pcol unused)
+  // PageRank: contributions live in the compacted space of non-dangling vertices
+  // (every column of an in-CSR is a page with out-links), cached per out_degree array
+  const int32_t *pr_od = nullptr;
+  int64_t pr_bc = 0;           // compact slots per rank block
+  inl::DevBuf pr_cidx;         // int32 [n_global]: exchange-space index, -1 if dangling
+  inl::DevBuf pr_col;          // int32 [nnz]: gather columns in the compact space (hot kept)
+  inl::DevBuf pr_hot;          // int32 [n_hot]: hot slots in the compact space
 };
 
 namespace inl {

@@ -3,6 +3,11 @@
 // rows; epilogue computes PR', the next contribution and the dangling partials)
 // + one single-CTA fixed-order reduction of the dangling partials.  On P > 1
 // ranks the contribution slice and the rank's dangling sum are allgathered.
+#include <cub/device/device_scan.cuh>
+
+#include <algorithm>
+#include <vector>
+
 #include "comm.h"
 #include "gather.cuh"
 
@@ -10,15 +15,15 @@ namespace inl {
 
 namespace {
 
-// c[v] = PR^0(v) / outdeg(v) with PR^0 = 1/n; dangling count for D^0.
-__global__ void k_pr_init(const int32_t *__restrict__ od, int64_t n, float *__restrict__ c,
-                          unsigned long long *__restrict__ n_dangling) {
+// c[cidx(v)] = PR^0(v) / outdeg(v) with PR^0 = 1/n; dangling count for D^0.
+__global__ void k_pr_init(const int32_t *__restrict__ od, const int32_t *__restrict__ cidx, int64_t n,
+                          float *__restrict__ c, unsigned long long *__restrict__ n_dangling) {
   const float pr0 = (float)(1.0 / (double)n);
   unsigned long long cnt = 0;
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
        v += (int64_t)gridDim.x * blockDim.x) {
     const int d = od[v];
-    c[v] = d > 0 ? pr0 / (float)d : 0.0f;
+    if (d > 0) c[cidx[v]] = pr0 / (float)d;
     cnt += d == 0;
   }
   for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
@@ -61,6 +66,47 @@ __global__ void k_fill(float *__restrict__ a, int64_t n, float v) {
     a[i] = v;
 }
 
+// ---- compaction of the contribution space to pages with out-links ----
+__global__ void k_nd_flags(const int32_t *__restrict__ od, int64_t n, int32_t *__restrict__ f) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n;
+       v += (int64_t)gridDim.x * blockDim.x)
+    f[v] = v < n && od[v] > 0;
+}
+
+// exchange-space index: block q = v / B holds slots [q*Bc, (q+1)*Bc); -1 for dangling pages
+__global__ void k_cidx(const int32_t *__restrict__ od, const int32_t *__restrict__ pos, int64_t n, int64_t B,
+                       int64_t Bc, int32_t *__restrict__ cidx) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t q = v / B;
+    cidx[v] = od[v] > 0 ? (int32_t)(q * Bc + (pos[v] - pos[q * B])) : -1;
+  }
+}
+
+// gather columns in the compact space (hot slots kept); a column without out-links
+// (inconsistent input) reads the zero slot
+__global__ void k_remap_cols(const int32_t *__restrict__ col, int64_t nnz, const int32_t *__restrict__ cidx,
+                             int32_t zero_slot, int32_t *__restrict__ out) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = col[k];
+    if (c < 0) {
+      out[k] = c;
+    } else {
+      const int32_t m = cidx[c];
+      out[k] = m >= 0 ? m : zero_slot;
+    }
+  }
+}
+
+__global__ void k_remap_hot(const int32_t *__restrict__ hot, int n_hot, const int32_t *__restrict__ cidx,
+                            int32_t zero_slot, int32_t *__restrict__ out) {
+  for (int h = blockIdx.x * blockDim.x + threadIdx.x; h < n_hot; h += gridDim.x * blockDim.x) {
+    const int32_t m = cidx[hot[h]];
+    out[h] = m >= 0 ? m : zero_slot;
+  }
+}
+
 int grid_for(int64_t n, int sms) {
   int64_t g = (n + 255) / 256;
   if (g > (int64_t)sms * 16) g = (int64_t)sms * 16;
@@ -68,6 +114,43 @@ int grid_for(int64_t n, int sms) {
 }
 
 }  // namespace
+
+// Compact (exchange-space) numbering of the pages with out-links, the gather columns in
+// that space, and the slots per rank block.  Cached in the plan per out_degree array.
+static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, int P) {
+  if (p->pr_od == od) return;
+  cudaStream_t st = ctx->stream;
+  const int64_t n = p->n_global;
+  int32_t *flags = (int32_t *)ctx->s_e.get(sizeof(int32_t) * (n + 1));
+  int32_t *pos = (int32_t *)ctx->s_f.get(sizeof(int32_t) * (n + 1));
+  k_nd_flags<<<grid_for(n + 1, ctx->num_sms), 256, 0, st>>>(od, n, flags);
+  size_t need = 0;
+  INL_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, need, flags, pos, n + 1, st));
+  INL_CUDA(cub::DeviceScan::ExclusiveSum(ctx->s_tmp.get(need), need, flags, pos, n + 1, st));
+  std::vector<int32_t> at(P + 1);
+  for (int q = 0; q <= P; ++q) {
+    const int64_t v = std::min<int64_t>((int64_t)q * B, n);
+    INL_CUDA(cudaMemcpyAsync(&at[q], pos + v, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  }
+  INL_CUDA(cudaStreamSynchronize(st));
+  int64_t bc = 1;
+  for (int q = 0; q < P; ++q) bc = std::max<int64_t>(bc, (int64_t)at[q + 1] - at[q]);
+  p->pr_bc = bc;
+  int32_t *cidx = (int32_t *)p->pr_cidx.get(sizeof(int32_t) * (n > 0 ? n : 1));
+  k_cidx<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, pos, n, B, bc, cidx);
+  const int32_t zero_slot = (int32_t)(bc * P);
+  const int32_t *src = p->n_hot > 0 ? (const int32_t *)p->pcol.p : p->col_idx;
+  int32_t *pc = (int32_t *)p->pr_col.get(sizeof(int32_t) * (p->nnz > 0 ? p->nnz : 1));
+  if (p->nnz > 0)
+    k_remap_cols<<<grid_for(p->nnz, ctx->num_sms), 256, 0, st>>>(src, p->nnz, cidx, zero_slot, pc);
+  if (p->n_hot > 0) {
+    int32_t *ph = (int32_t *)p->pr_hot.get(sizeof(int32_t) * p->n_hot);
+    k_remap_hot<<<grid_for(p->n_hot, ctx->num_sms), 256, 0, st>>>((const int32_t *)p->hot_cols.p, (int)p->n_hot,
+                                                                 cidx, zero_slot, ph);
+  }
+  INL_CUDA(cudaGetLastError());
+  p->pr_od = od;
+}
 
 void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damping, int iters,
                   float *rank) {
@@ -81,10 +164,16 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
   }
   const int P = ctx->nranks;
   const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
-  const int64_t B = DIST ? (n + P - 1) / P : n;  // allgather block (inl_partition_rows)
+  const int64_t B = DIST ? (n + P - 1) / P : n;  // row block (inl_partition_rows)
   const int64_t npad = B * P;
-  float *c_cur = (float *)ctx->s_a.get(sizeof(float) * npad);
-  float *c_next = (float *)ctx->s_b.get(sizeof(float) * npad);
+  pr_compact(ctx, p, out_degree, B, DIST ? P : 1);
+  const int64_t Bc = p->pr_bc;                    // compact slots per block (exchange count)
+  const int64_t ncomp = Bc * (DIST ? P : 1) + 1;  // + the zero slot
+  float *c_cur = (float *)ctx->s_a.get(sizeof(float) * ncomp);
+  float *c_next = (float *)ctx->s_b.get(sizeof(float) * ncomp);
+  INL_CUDA(cudaMemsetAsync(c_cur, 0, sizeof(float) * ncomp, st));
+  INL_CUDA(cudaMemsetAsync(c_next, 0, sizeof(float) * ncomp, st));
+  const int32_t *cidx = (const int32_t *)p->pr_cidx.p;
   char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (P + 1));
   float *base = (float *)scal;
   unsigned long long *ndang = (unsigned long long *)(scal + 8);
@@ -94,7 +183,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
   if (DIST) rank_pad = (float *)ctx->s_d.get(sizeof(float) * npad);
 
   INL_CUDA(cudaMemsetAsync(ndang, 0, sizeof(unsigned long long), st));
-  k_pr_init<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(out_degree, n, c_cur, ndang);
+  k_pr_init<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(out_degree, cidx, n, c_cur, ndang);
   k_pr_base0<<<1, 1, 0, st>>>(ndang, n, (double)damping, base);
   INL_CUDA(cudaGetLastError());
 
@@ -104,14 +193,15 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
     const bool last = t + 1 == iters;
     GatherArgs a{p->row_ptr, p->col_idx, nullptr, c_cur, p->nnz, p->n_rows,
                  p->bins.t_thread, p->bins.t_warp, p->bins.t_block, p->bins.grid_chunk, false};
-    PrEpi epi{out_degree, c_next, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
+    PrEpi epi{out_degree, c_next, cidx, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
               p->row_begin, 0.0f};
-    launch_gather<false>(ctx, p, a, epi, dpart);
+    launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p,
+                         p->n_hot > 0 ? (const int32_t *)p->pr_hot.p : nullptr);
     if (!last) {
       k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
       INL_CUDA(cudaGetLastError());
       if (DIST) {
-        comm_allgather(ctx, c_next + (int64_t)ctx->rank * B, c_next, B, ncclFloat32, dloc, dall);
+        comm_allgather(ctx, c_next + (int64_t)ctx->rank * Bc, c_next, Bc, ncclFloat32, dloc, dall);
       }
       k_pr_base<<<1, 1, 0, st>>>(dall, P, n, (double)damping, base);
       INL_CUDA(cudaGetLastError());

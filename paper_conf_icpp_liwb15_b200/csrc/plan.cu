@@ -224,6 +224,7 @@ void build_plan(inl_plan p) {
   const int64_t n = p->n_rows;
   const Bins &b = p->bins;
   p->info.bins = {b.t_thread, b.t_warp, b.t_block, b.grid_chunk, b.cta, b.flags};
+  p->pr_od = nullptr;  // PageRank compaction is rebuilt for a (re)built plan
   p->n_tiles = p->n_long = p->n_chunks = 0;
   if (n == 0) return;
   INL_CHECK(n < INT32_MAX, "plan: n_rows must be < 2^31");

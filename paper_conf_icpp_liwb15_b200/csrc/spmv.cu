@@ -11,11 +11,11 @@ __global__ void k_build_xhot(const float *__restrict__ x, const int32_t *__restr
 }
 }  // namespace
 
-void build_xhot(inl_ctx ctx, inl_plan p, const float *x) {
+void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols) {
   if (p->n_hot == 0) return;
   const int n = (int)p->n_hot;
-  k_build_xhot<<<(n + 255) / 256, 256, 0, ctx->stream>>>(x, (const int32_t *)p->hot_cols.p, n,
-                                                          (float *)p->x_hot.p);
+  k_build_xhot<<<(n + 255) / 256, 256, 0, ctx->stream>>>(
+      x, hot_cols ? hot_cols : (const int32_t *)p->hot_cols.p, n, (float *)p->x_hot.p);
   INL_CUDA(cudaGetLastError());
 }
 
