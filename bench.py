@@ -209,10 +209,15 @@ def run_inl(a):
         bytes_local = pagerank_bytes_per_iter(nnz_local, A.n_rows, A.n_global) * a.iterations
         launches_per_step = 3 + 4 * a.iterations  # init; per iteration xhot + gather + dsum + base
     else:
-        srcs = inlgen.sources(g["row_ptr"].cpu().numpy(), 8) if world == 1 else [0]
+        # seeded sources of degree > 0 (+ the max-degree vertex); under torchrun rank 0 picks
+        # them from its row block (global ids: its row_begin is 0) and broadcasts them
+        srcs = inlgen.sources(g["row_ptr"].cpu().numpy(), 8) if rank == 0 else []
         if world > 1:
-            src_t = torch.tensor(srcs, device="cuda")
+            src_t = torch.full((16,), -1, dtype=torch.int64, device="cuda")
+            if rank == 0:
+                src_t[:len(srcs)] = torch.tensor(srcs, dtype=torch.int64)
             dist.broadcast(src_t, 0)
+            srcs = [int(v) for v in src_t.tolist() if v >= 0]
         out_arr = torch.empty(A.n_global, dtype=torch.int32, device="cuda")
         state = {"i": 0, "last": None}
 
