@@ -123,56 +123,29 @@ struct GatherPlan {
 
 // x[c] for a remapped column: hot slots (c = 0x80000000 | slot) from shared memory at
 // xs + (c << 2) (the shift drops the tag bit), cold columns from global memory
-// (read-only path).  One predicated load of each kind and a select: branch-free.
-__device__ __forceinline__ float gx(int32_t c, bool in, uint32_t xs_base, const float *x) {
-  float r;
-  asm("{\n\t"
-      ".reg .pred h, g, i;\n\t"
-      ".reg .b32 sa;\n\t"
-      ".reg .b64 ga;\n\t"
-      ".reg .f32 hv, cv;\n\t"
-      "setp.ne.b32 i, %2, 0;\n\t"
-      "setp.lt.and.s32 h, %1, 0, i;\n\t"
-      "setp.ge.and.s32 g, %1, 0, i;\n\t"
-      "shl.b32 sa, %1, 2;\n\t"
-      "add.u32 sa, sa, %3;\n\t"
-      "mov.f32 hv, 0f00000000;\n\t"
-      "mov.f32 cv, 0f00000000;\n\t"
-      "@h ld.shared.f32 hv, [sa];\n\t"
-      "mad.wide.s32 ga, %1, 4, %4;\n\t"
-      "@g ld.global.nc.f32 cv, [ga];\n\t"
-      "selp.f32 %0, hv, cv, h;\n\t"
-      "}"
-      : "=f"(r)
-      : "r"(c), "r"((int)in), "r"(xs_base), "l"(x));
-  return r;
-}
-
-// gx for an entry known to be inside the item (no `in` predicate).
-__device__ __forceinline__ float gx_in(int32_t c, uint32_t xs_base, const float *x) {
+// (read-only path).  Two complementary predicated loads into ONE register: no select.
+__device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x) {
   float r;
   asm("{\n\t"
       ".reg .pred h;\n\t"
       ".reg .b32 sa;\n\t"
       ".reg .b64 ga;\n\t"
-      ".reg .f32 hv, cv;\n\t"
       "setp.lt.s32 h, %1, 0;\n\t"
       "shl.b32 sa, %1, 2;\n\t"
       "add.u32 sa, sa, %2;\n\t"
-      "mov.f32 hv, 0f00000000;\n\t"
-      "mov.f32 cv, 0f00000000;\n\t"
-      "@h ld.shared.f32 hv, [sa];\n\t"
       "mad.wide.s32 ga, %1, 4, %3;\n\t"
-      "@!h ld.global.nc.f32 cv, [ga];\n\t"
-      "selp.f32 %0, hv, cv, h;\n\t"
+      "@h ld.shared.f32 %0, [sa];\n\t"
+#if defined(INL_GX_NA)
+      "@!h ld.global.nc.L1::no_allocate.f32 %0, [ga];\n\t"
+#elif defined(INL_GX_CG)
+      "@!h ld.global.cg.f32 %0, [ga];\n\t"
+#else
+      "@!h ld.global.nc.f32 %0, [ga];\n\t"
+#endif
       "}"
       : "=f"(r)
       : "r"(c), "r"(xs_base), "l"(x));
   return r;
-}
-
-__device__ __forceinline__ float lval(const float *val, int64_t k, bool in) {
-  return val ? __uint_as_float(ld_stream_pred(val + k, in)) : (in ? 1.0f : 0.0f);
 }
 
 // L2 prefetch of entries [lo, hi) of the col/val streams (short range: one pass ahead keeps
@@ -189,35 +162,52 @@ __device__ __forceinline__ void prefetch_item(const GatherArgs &a, const WorkIte
   if (it.j < 0) prefetch_span(a.row_ptr + it.r0, a.row_ptr + it.r1 + 1, a.row_ptr + a.n_rows + 1);
 }
 
-// Stream registers of one pass: lane l holds entries q0 .. q0+E-1 of the item span.
+// Stream registers of one pass: lane l holds the (remapped) columns of entries
+// q0 .. q0+E-1 of the item span and the 32-bit word of the row-start bit array that
+// covers them (double-buffered: they feed the gathers); the values are single-buffered
+// (loaded once the current pass's products are formed).
 template <int E>
-struct PassRegs {
+struct ColRegs {
   uint32_t cv[E];
-  float vv[E];
+  uint32_t fw;
 };
 
-template <int E, bool VALS>
-__device__ __forceinline__ void load_pass(const GatherArgs &a, int64_t s, int len, int q0, PassRegs<E> &r) {
-  const int64_t k0 = s + q0;  // E-aligned; the group lies inside the arrays unless at the end
+// Lanes whose group lies wholly outside the item load nothing (their entries are masked
+// before use).
+template <int E>
+__device__ __forceinline__ void load_cols(const GatherArgs &a, const uint32_t *rs_bits, int64_t s, int len,
+                                          int q0, ColRegs<E> &r) {
+  const int64_t k0 = s + q0;  // E-aligned, >= 0
+  if (q0 >= len || q0 + E <= 0) return;
+  r.fw = __ldg(rs_bits + (k0 >> 5));
   if (a.vec && k0 + E <= a.nnz) {
 #pragma unroll
     for (int h = 0; h < E / 8; ++h) {
       const U32x8 c = ld_stream_256(a.col_idx + k0 + 8 * h);
 #pragma unroll
       for (int j = 0; j < 8; ++j) r.cv[8 * h + j] = c.v[j];
-      if (VALS) {
-        const U32x8 v = ld_stream_256(a.val + k0 + 8 * h);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) r.vv[8 * h + j] = __uint_as_float(v.v[j]);
-      }
     }
   } else {
 #pragma unroll
-    for (int j = 0; j < E; ++j) {
-      const bool in = (unsigned)(q0 + j) < (unsigned)len;
-      r.cv[j] = ld_stream_pred(a.col_idx + k0 + j, in);
-      r.vv[j] = VALS ? __uint_as_float(ld_stream_pred(a.val + k0 + j, in)) : 0.0f;
+    for (int j = 0; j < E; ++j) r.cv[j] = ld_stream_pred(a.col_idx + k0 + j, (unsigned)(q0 + j) < (unsigned)len);
+  }
+}
+
+template <int E>
+__device__ __forceinline__ void load_vals(const GatherArgs &a, int64_t s, int len, int q0, float (&vv)[E]) {
+  const int64_t k0 = s + q0;
+  if (q0 >= len || q0 + E <= 0) return;
+  if (a.vec && k0 + E <= a.nnz) {
+#pragma unroll
+    for (int h = 0; h < E / 8; ++h) {
+      const U32x8 v = ld_stream_256(a.val + k0 + 8 * h);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) vv[8 * h + j] = __uint_as_float(v.v[j]);
     }
+  } else {
+#pragma unroll
+    for (int j = 0; j < E; ++j)
+      vv[j] = __uint_as_float(ld_stream_pred(a.val + k0 + j, (unsigned)(q0 + j) < (unsigned)len));
   }
 }
 
@@ -241,10 +231,13 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
   if (lane == 0 && gw < gp.n_items) prefetch_item<VALS>(a, gp.items[gw]);
   for (int i = threadIdx.x * 4; i < gp.n_hot; i += NWARP * 32 * 4)
     *reinterpret_cast<float4 *>(xs + i) = __ldg(reinterpret_cast<const float4 *>(gp.x_hot + i));
+  if (threadIdx.x == 0) xs[gp.n_hot] = 0.0f;  // the zero slot (masked entries gather it)
   __syncthreads();
   epi.init();
   const uint32_t xs_base = smem_u32(xs);
+  const uint32_t ZS = 0x80000000u | (uint32_t)gp.n_hot;  // remapped column of the zero slot
   const unsigned lt = (1u << lane) - 1u;
+  const unsigned le = 0xffffffffu >> (31 - lane);
   if (gw >= gp.n_items) return;
 
   // dynamic schedule: a warp's first item is gw, later ones come from the work counter
@@ -255,36 +248,38 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
     t = __shfl_sync(0xffffffffu, t, 0);
     return (int)min(t + (unsigned long long)nwarps, (unsigned long long)gp.n_items);
   };
-  // pipeline: `nx` holds the stream registers of the pass after the current one
   int idx = gw;
   WorkItem it = gp.items[idx];
   int nidx = grab();
-  WorkItem itn;  // the next item's descriptor (prefetched)
-  if (nidx < gp.n_items) itn = gp.items[nidx];
-  PassRegs<E> nx;
-  load_pass<E, VALS>(a, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, nx);
+  int64_t ns = 0, ne = 0;  // the next item's span (its full descriptor is re-read at the switch)
+  if (nidx < gp.n_items) {
+    ns = gp.items[nidx].s;
+    ne = gp.items[nidx].e;
+  }
+  // column registers of the next pass (a pass copies them, then refills them with the
+  // loads of the pass after it); one value set (reloaded once a pass's products are formed)
+  ColRegs<E> nx;
+  float vv[E];
+  load_cols<E>(a, gp.rs_bits, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, nx);
+  if (VALS) load_vals<E>(a, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, vv);
   for (;;) {
     const int64_t s = it.s;
     const int len = (int)(it.e - s);
     const bool has_next = nidx < gp.n_items;
-    if (lane == 0 && has_next) prefetch_item<VALS>(a, itn);
+    const bool chunk = it.j >= 0;
+    if (lane == 0 && has_next) prefetch_item<VALS>(a, gp.items[nidx]);
     double dacc = 0.0;
     int nnzr = 0;
-    if (it.j < 0) {  // tile: non-empty rows -> (offset, row) lists; empty rows finish here (y = 0)
+    if (!chunk) {  // tile: non-empty rows -> list; empty rows finish here (y = 0)
       const int nr = it.r1 - it.r0;
-      for (int rb = 0; rb < nr; rb += 32) {
-        const int r = rb + lane;
-        int off = 0, d = 0;
-        if (r < nr) {
-          const int64_t b = __ldg(a.row_ptr + it.r0 + r);
-          off = (int)(b - s);
-          d = (int)(__ldg(a.row_ptr + it.r0 + r + 1) - b);
-        }
+      for (int rb0 = 0; rb0 < nr; rb0 += 32) {
+        const int r = rb0 + lane;
+        int d = 0;
+        if (r < nr) d = (int)(__ldg(a.row_ptr + it.r0 + r + 1) - __ldg(a.row_ptr + it.r0 + r));
         const unsigned nz = __ballot_sync(0xffffffffu, r < nr && d > 0);
         if (r < nr && d > 0) ws.nzrow[nnzr + __popc(nz & lt)] = (short)r;
         if (r < nr && d == 0) dacc += epi(it.r0 + r, 0.0f);
         nnzr += __popc(nz);
-        (void)off;
       }
     } else {  // a chunk is one row: its only start is offset 0
       if (lane == 0) ws.nzrow[0] = 0;
@@ -293,94 +288,104 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
     int kcur = 0;        // number of row starts consumed so far in this item
     int open_row = -1;   // local row open across the pass boundary
     float carry = 0.0f;  // its partial sum
+
     for (int p0 = first_p0<E>(it);; p0 += P) {  // >= 1 pass: it also hands the pipeline over
+      ColRegs<E> cur = nx;
       const int q0 = p0 + E * lane;
-      // (A) gathers of the current pass (its stream registers were loaded one pass ago)
+      const bool more = p0 + P < len;
+      // (1) the next pass's columns (same item, or the next item's first pass)
+      if (more) load_cols<E>(a, gp.rs_bits, s, len, q0 + P, nx);
+      else if (has_next)
+        load_cols<E>(a, gp.rs_bits, ns, (int)(ne - ns), -(int)(ns & (E - 1)) + E * lane, nx);
+      // (2) my E row-start flags; entries outside the item gather the zero slot
+      unsigned fl = (cur.fw >> (int)((s + q0) & 31)) & EM;
+      if (!(p0 >= 0 && p0 + P <= len)) {  // edge pass of the item (warp-uniform)
+        const int lo = q0 < 0 ? -q0 : 0, hi = len - q0 < E ? len - q0 : E;
+        fl = (lo < hi && hi > 0 && lo < E) ? fl & (EM << lo) & (EM >> (E - hi)) : 0u;
+#pragma unroll
+        for (int j = 0; j < E; ++j) {
+          if ((unsigned)(q0 + j) >= (unsigned)len) {
+            cur.cv[j] = ZS;
+            vv[j] = 0.0f;
+          }
+        }
+      }
+      if (chunk && q0 <= 0 && q0 + E > 0) fl |= 1u << (-q0);  // a chunk (re)starts its row
+      // (3) gathers
       float pr[E];
-      if (q0 >= 0 && q0 + E <= len) {  // whole group inside the item: no per-entry predicates
-#pragma unroll
-        for (int j = 0; j < E; ++j) {
-          const float xv = gx_in((int32_t)nx.cv[j], xs_base, a.x);
-          pr[j] = VALS ? nx.vv[j] * xv : xv;
-        }
-      } else {
-#pragma unroll
-        for (int j = 0; j < E; ++j) {
-          const bool in = (unsigned)(q0 + j) < (unsigned)len;
-          const float xv = gx((int32_t)nx.cv[j], in, xs_base, a.x);
-          pr[j] = in ? (VALS ? nx.vv[j] * xv : xv) : 0.0f;
-        }
-      }
-      // issue the next pass's stream loads now (same item or the next item's first pass)
-      if (p0 + P < len) {
-        load_pass<E, VALS>(a, s, len, q0 + P, nx);
-      } else if (has_next) {
-        load_pass<E, VALS>(a, itn.s, (int)(itn.e - itn.s), first_p0<E>(itn) + E * lane, nx);
-      }
-      // my E row-start flags (plan bit array; my segment is E-aligned within a 32-bit word)
-      unsigned fl = 0u;
-      {
-        const int64_t k0 = s + q0;  // E-aligned
-        if (q0 + E > 0 && q0 < len) {
-          const uint32_t wv = __ldg(gp.rs_bits + (k0 >> 5));
-          fl = (wv >> ((int)(k0 & 31))) & EM;
-          const int lo = q0 < 0 ? -q0 : 0, hi = len - q0 < E ? len - q0 : E;
-          fl &= (EM << lo) & (EM >> (E - hi));  // entries of this item only
-          if (it.j >= 0 && q0 <= 0) fl |= 1u << lo;  // a chunk (re)starts its row at offset 0
-        }
-      }
-      // number of starts before my segment: exclusive scan of popc(fl)
-      int before = __popc(fl);
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const int t = __shfl_up_sync(0xffffffffu, before, d);
-        if (lane >= d) before += t;
-      }
-      const int kpass = kcur;
-      kcur += __shfl_sync(0xffffffffu, before, 31);
-      before -= __popc(fl);
-      // THREAD-mapped rows: complete inside my segment -> emitted here
-      float head = 0.0f, cur = 0.0f;
-      int rank = before - 1;
 #pragma unroll
       for (int j = 0; j < E; ++j) {
-        if (fl & (1u << j)) {
-          if (rank < before) head = cur;  // first start: what came before belongs to the open row
-          else dacc += epi(it.r0 + ws.nzrow[kpass + rank], cur);
-          ++rank;
-          cur = 0.0f;
-        }
-        cur += pr[j];
+        const float xv = gx((int32_t)cur.cv[j], xs_base, a.x);
+        pr[j] = VALS ? vv[j] * xv : xv;
       }
-      const bool F = fl != 0u;
-      if (!F) head = cur;
-      // WARP-mapped rows: segmented inclusive scan of (F ? tail : head) across lanes
-      float S = F ? cur : (lane == 0 ? head + carry : head);
-      bool G = F;
+      if (VALS) {  // the next pass's values
+        if (more) load_vals<E>(a, s, len, q0 + P, vv);
+        else if (has_next) load_vals<E>(a, ns, (int)(ne - ns), -(int)(ns & (E - 1)) + E * lane, vv);
+      }
+      const int nf = __popc(fl);
+      const unsigned fmask = __ballot_sync(0xffffffffu, nf != 0);
+      const int kpass = kcur;
+      float head = 0.0f, tail = 0.0f;
+      int before;
+      if (__any_sync(0xffffffffu, nf >= 2)) {
+        // THREAD-mapped rows complete inside my segment are emitted here
+        before = nf;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const int t = __shfl_up_sync(0xffffffffu, before, d);
+          if (lane >= d) before += t;
+        }
+        kcur += __shfl_sync(0xffffffffu, before, 31);
+        before -= nf;
+        int rank = before - 1;
+#pragma unroll
+        for (int j = 0; j < E; ++j) {
+          if (fl & (1u << j)) {
+            if (rank < before) head = tail;  // first start: what came before belongs to the open row
+            else dacc += epi(it.r0 + ws.nzrow[kpass + rank], tail);
+            ++rank;
+            tail = 0.0f;
+          }
+          tail += pr[j];
+        }
+        if (!fl) head = tail;
+      } else {  // at most one start per lane (warp-bin rows and chunks): one serial chain
+        before = __popc(fmask & lt);
+        kcur += __popc(fmask);
+#pragma unroll
+        for (int j = 0; j < E; ++j) {
+          const bool f = (fl >> j) & 1u;
+          if (f) head = tail;
+          tail = (f ? 0.0f : tail) + pr[j];
+        }
+        if (!fl) head = tail;
+      }
+      // WARP-mapped rows: segmented inclusive scan across lanes; a segment starts at the
+      // last lane <= me holding a start (span = lanes below me in my segment)
+      if (lane == 0) head += carry;
+      const bool F = nf != 0;
+      float S = F ? tail : head;
+      const unsigned hm = fmask & le;
+      const int span = hm ? lane - (31 - __clz(hm)) : lane;
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) {
         const float t = __shfl_up_sync(0xffffffffu, S, d);
-        const bool tg = __shfl_up_sync(0xffffffffu, G, d);
-        if (lane >= d) {
-          if (!G) S += t;
-          G = G || tg;
-        }
+        if (span >= d) S += t;
       }
       float Ein = __shfl_up_sync(0xffffffffu, S, 1);  // value entering my segment
-      if (lane == 0) Ein = carry;
-      if (F) {  // the row open at my segment start ends at my first flag
+      if (lane == 0) Ein = 0.0f;
+      if (F) {  // the row open at my segment start ends at my first start
         const int rr = before > 0 ? ws.nzrow[kpass + before - 1] : open_row;
         if (rr >= 0) dacc += epi(it.r0 + rr, Ein + head);
       }
-      const unsigned anyF = __ballot_sync(0xffffffffu, F);
       carry = __shfl_sync(0xffffffffu, S, 31);
-      if (anyF) open_row = ws.nzrow[it.j < 0 ? kcur - 1 : 0];
-      __syncwarp();
-      if (p0 + P >= len) break;
+      if (fmask) open_row = ws.nzrow[chunk ? 0 : kcur - 1];
+      if (!more) break;
     }
+    __syncwarp();
     // the row still open at the end of the item
     if (lane == 0 && open_row >= 0) {
-      if (it.j < 0 || it.nch == 1) {
+      if (!chunk || it.nch == 1) {
         dacc += epi(it.r0 + open_row, carry);
       } else {  // grid bin: partial of chunk c; the last chunk to finish combines in order
         gp.partials[it.pbase + it.c] = carry;
@@ -403,9 +408,12 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
     __syncwarp();
     if (!has_next) break;
     idx = nidx;
-    it = itn;
+    it = gp.items[idx];
     nidx = grab();
-    if (nidx < gp.n_items) itn = gp.items[nidx];
+    if (nidx < gp.n_items) {
+      ns = gp.items[nidx].s;
+      ne = gp.items[nidx].e;
+    }
   }
 }
 

@@ -18,7 +18,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libinl.so")
+LIB_PATH = os.environ.get("INL_LIB") or os.path.join(_HERE, "libinl.so")  # INL_LIB: A/B variant builds
 
 INL_OK = 0
 STATUS = {0: "INL_OK", 1: "INL_ERR_INVALID_ARGUMENT", 2: "INL_ERR_OUT_OF_MEMORY", 3: "INL_ERR_CUDA",

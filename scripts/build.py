@@ -66,9 +66,11 @@ def build_inlgen(force: bool = False) -> str:
     return out
 
 
-def build_inl(force: bool = False) -> str:
+def build_inl(force: bool = False, defines: list[str] | None = None, out: str | None = None) -> str:
+    """defines/out: an experiment variant (-D flags) written to another path (A/B runs
+    select it with INL_LIB=<path>); the product build uses neither."""
     pkg = os.path.join(ROOT, "paper_conf_icpp_liwb15_b200")
-    out = os.path.join(pkg, "libinl.so")
+    out = out or os.path.join(pkg, "libinl.so")
     csrc = os.path.join(pkg, "csrc")
     srcs = sorted(glob.glob(os.path.join(csrc, "*.cu")) + glob.glob(os.path.join(csrc, "*.cpp")))
     deps = srcs + glob.glob(os.path.join(csrc, "*.cuh")) + glob.glob(os.path.join(csrc, "*.h")) + \
@@ -77,7 +79,9 @@ def build_inl(force: bool = False) -> str:
         raise RuntimeError("no sources under " + csrc)
     if force or _stale(out, deps):
         nccl = _nccl_dir()
-        _run([NVCC] + NVCC_COMMON + ["-Xptxas", "-v" if os.environ.get("INL_PTXAS_V") else "-O3",
+        os.makedirs(os.path.dirname(out), exist_ok=True)
+        _run([NVCC] + NVCC_COMMON + ["-D" + d for d in (defines or [])] +
+             ["-Xptxas", "-v" if os.environ.get("INL_PTXAS_V") else "-O3",
                                      "-I", os.path.join(nccl, "include"), "-I", os.path.join(ROOT, "include"),
                                      "-shared", "-o", out] + srcs +
              ["-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
@@ -100,7 +104,13 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("--only", choices=["oracle", "inlgen", "inl"])
+    ap.add_argument("--variant", nargs="+", metavar="NAME [DEFINE ...]",
+                    help="build an experiment variant build/variants/libinl_NAME.so with -D DEFINEs")
     a = ap.parse_args()
+    if a.variant:
+        o = build_inl(True, a.variant[1:], os.path.join(ROOT, "build", "variants", f"libinl_{a.variant[0]}.so"))
+        print("built", o)
+        sys.exit(0)
     for o in build_all(a.force, a.only):
         print("built", o)
     sys.exit(0)
