@@ -123,7 +123,8 @@ struct GatherPlan {
 
 // x[c] for a remapped column: hot slots (c = 0x80000000 | slot) from shared memory at
 // xs + (c << 2) (the shift drops the tag bit), cold columns from global memory
-// (read-only path).  Two complementary predicated loads into ONE register: no select.
+// (ld.global.cg: cold columns have no L1 reuse).  Two complementary predicated loads into
+// ONE register: no select.
 __device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x) {
   float r;
   asm("{\n\t"
@@ -137,10 +138,10 @@ __device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x)
       "@h ld.shared.f32 %0, [sa];\n\t"
 #if defined(INL_GX_NA)
       "@!h ld.global.nc.L1::no_allocate.f32 %0, [ga];\n\t"
-#elif defined(INL_GX_CG)
-      "@!h ld.global.cg.f32 %0, [ga];\n\t"
-#else
+#elif defined(INL_GX_NC)
       "@!h ld.global.nc.f32 %0, [ga];\n\t"
+#else  // cache-global (L2 only): measured 4% faster than the read-only path (profiles/r01)
+      "@!h ld.global.cg.f32 %0, [ga];\n\t"
 #endif
       "}"
       : "=f"(r)
