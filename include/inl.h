@@ -151,6 +151,16 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
                    inl_stats *stats, inl_plan plan);
 
+/* Kernel timer (measurement only; off by default).  While enabled, every launch of the
+ * path's main kernels ("k_gather", "k_gather_thread_only", "k_expand_flat",
+ * "k_expand_grid", "k_bfs_bottom_up") is bracketed by CUDA events recorded on the ctx
+ * stream — stream-ordered, so the asynchronous SpMV / PageRank calls stay asynchronous.
+ * inl_ktimer_enable(ctx, 1) clears the counters; inl_ktimer_read synchronizes the ctx
+ * stream and returns, for the named kernel, the number of launches and the summed
+ * device duration in ms (0 / 0 if it never ran).  Unknown names are not an error. */
+inl_status inl_ktimer_enable(inl_ctx ctx, int32_t enable);
+inl_status inl_ktimer_read(inl_ctx ctx, const char *kernel, int64_t *launches, double *total_ms);
+
 #ifdef __cplusplus
 }
 #endif

@@ -40,6 +40,53 @@ void DevBuf::release() {
   bytes = 0;
 }
 
+KTimer::Slot &KTimer::slot(const char *name) {
+  for (auto &s : slots)
+    if (s.name == name) return s;
+  slots.emplace_back();
+  slots.back().name = name;
+  return slots.back();
+}
+
+cudaEvent_t KTimer::ev() {
+  if (pool.empty()) {
+    cudaEvent_t e;
+    INL_CUDA(cudaEventCreate(&e));
+    return e;
+  }
+  cudaEvent_t e = pool.back();
+  pool.pop_back();
+  return e;
+}
+
+void KTimer::resolve() {
+  for (auto &s : slots) {
+    for (auto &pr : s.pending) {
+      float ms = 0.0f;
+      INL_CUDA(cudaEventElapsedTime(&ms, pr.first, pr.second));
+      s.ms += ms;
+      s.launches += 1;
+      pool.push_back(pr.first);
+      pool.push_back(pr.second);
+    }
+    s.pending.clear();
+  }
+}
+
+void KTimer::clear() {
+  for (auto &s : slots)
+    for (auto &pr : s.pending) {
+      pool.push_back(pr.first);
+      pool.push_back(pr.second);
+    }
+  slots.clear();
+}
+
+KTimer::~KTimer() {
+  clear();
+  for (cudaEvent_t e : pool) cudaEventDestroy(e);
+}
+
 Bins resolve_bins(const inl_bins *b) {
   Bins r{8, 1024, 16384, 4096, 256, 0};
   if (b) {
@@ -320,6 +367,33 @@ inl_status inl_ctx_destroy(inl_ctx ctx) {
   ctx->closed = true;
   if (ctx->live_plans == 0) free_ctx(ctx);
   return INL_OK;
+}
+
+inl_status inl_ktimer_enable(inl_ctx ctx, int32_t enable) {
+  if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
+  return guarded(ctx, [&] {
+    DeviceGuard g(ctx->device);
+    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx->ktimer.clear();
+    ctx->ktimer.on = enable != 0;
+  });
+}
+
+inl_status inl_ktimer_read(inl_ctx ctx, const char *kernel, int64_t *launches, double *total_ms) {
+  if (!ctx || !kernel || !launches || !total_ms)
+    return fail(ctx, INL_ERR_INVALID_ARGUMENT, "ktimer_read: NULL argument");
+  return guarded(ctx, [&] {
+    DeviceGuard g(ctx->device);
+    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx->ktimer.resolve();
+    *launches = 0;
+    *total_ms = 0.0;
+    for (auto &s : ctx->ktimer.slots)
+      if (s.name == kernel) {
+        *launches = s.launches;
+        *total_ms = s.ms;
+      }
+  });
 }
 
 inl_status inl_partition_rows(int64_t n, int32_t nranks, int64_t *bounds) {

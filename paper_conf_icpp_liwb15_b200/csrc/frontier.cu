@@ -468,12 +468,18 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
   ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
                f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
   if (nF > 0) {
-    if (b.flags & INL_BINS_THREAD_ONLY)  // the paper's baseline: thread-mapped, no balancing
+    if (b.flags & INL_BINS_THREAD_ONLY) {  // the paper's baseline: thread-mapped, no balancing
+      KScope ks(ctx, "k_expand");
       k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
-    else
+    } else {
+      KScope ks(ctx, "k_expand_flat");
       k_expand_flat<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
+    }
   }
-  k_expand_grid<Op><<<ctx->num_sms * 8, NT, 0, st>>>(a, op);
+  {
+    KScope ks(ctx, "k_expand_grid");
+    k_expand_grid<Op><<<ctx->num_sms * 8, NT, 0, st>>>(a, op);
+  }
   INL_CUDA(cudaGetLastError());
 }
 
@@ -634,8 +640,11 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           k_queue_to_bitmap<<<grid_for(nF, ctx->num_sms), 256, 0, st>>>(f.F, nF, fa);
         }
         INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
-        k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
-                                                         f.counts);
+        {
+          KScope ks(ctx, "k_bfs_bottom_up");
+          k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
+                                                           f.counts);
+        }
         INL_CUDA(cudaGetLastError());
         nF = read_count(ctx, f.counts);
         std::swap(fa, fb);

@@ -116,6 +116,7 @@ struct GatherPlan {
   const float *x_hot;   // [n_hot]
   int n_hot;
   const uint32_t *rs_bits;  // [nnz/32 + 1] bit k set iff entry k starts a non-empty row
+  const uint32_t *tile_nz;  // [n_tiles * 8] non-empty-row masks of the tiles
   unsigned long long *ticket;  // work counter (monotone across launches)
   unsigned long long base;     // its value at the start of this launch
 };
@@ -125,7 +126,7 @@ struct GatherPlan {
 // xs + (c << 2) (the shift drops the tag bit), cold columns from global memory
 // (ld.global.cg: cold columns have no L1 reuse).  Two complementary predicated loads into
 // ONE register: no select.
-__device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x) {
+__device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x, uint64_t pol) {
   float r;
   asm("{\n\t"
       ".reg .pred h;\n\t"
@@ -140,12 +141,14 @@ __device__ __forceinline__ float gx(int32_t c, uint32_t xs_base, const float *x)
       "@!h ld.global.nc.L1::no_allocate.f32 %0, [ga];\n\t"
 #elif defined(INL_GX_NC)
       "@!h ld.global.nc.f32 %0, [ga];\n\t"
+#elif defined(INL_GX_EL)
+      "@!h ld.global.cg.L2::cache_hint.f32 %0, [ga], %4;\n\t"
 #else  // cache-global (L2 only): measured 4% faster than the read-only path (profiles/r01)
       "@!h ld.global.cg.f32 %0, [ga];\n\t"
 #endif
       "}"
       : "=f"(r)
-      : "r"(c), "r"(xs_base), "l"(x));
+      : "r"(c), "r"(xs_base), "l"(x), "l"(pol));
   return r;
 }
 
@@ -160,7 +163,6 @@ __device__ __forceinline__ void prefetch_entries(const GatherArgs &a, int64_t lo
 template <bool VALS>
 __device__ __forceinline__ void prefetch_item(const GatherArgs &a, const WorkItem &it) {
   prefetch_entries<VALS>(a, it.s, min(it.e, it.s + 256));
-  if (it.j < 0) prefetch_span(a.row_ptr + it.r0, a.row_ptr + it.r1 + 1, a.row_ptr + a.n_rows + 1);
 }
 
 // Stream registers of one pass: lane l holds the (remapped) columns of entries
@@ -177,10 +179,10 @@ struct ColRegs {
 // before use).
 template <int E>
 __device__ __forceinline__ void load_cols(const GatherArgs &a, const uint32_t *rs_bits, int64_t s, int len,
-                                          int q0, ColRegs<E> &r) {
+                                          int q0, ColRegs<E> &r, uint64_t pol_ef) {
   const int64_t k0 = s + q0;  // E-aligned, >= 0
   if (q0 >= len || q0 + E <= 0) return;
-  r.fw = __ldg(rs_bits + (k0 >> 5));
+  r.fw = ld_stream_pol(rs_bits + (k0 >> 5), pol_ef);
   if (a.vec && k0 + E <= a.nnz) {
 #pragma unroll
     for (int h = 0; h < E / 8; ++h) {
@@ -237,6 +239,12 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
   epi.init();
   const uint32_t xs_base = smem_u32(xs);
   const uint32_t ZS = 0x80000000u | (uint32_t)gp.n_hot;  // remapped column of the zero slot
+  const uint64_t pol_ef = policy_evict_first();  // plan metadata streams (row-start bits, masks)
+#if defined(INL_GX_EL)
+  const uint64_t pol = policy_evict_last();
+#else
+  const uint64_t pol = 0;
+#endif
   const unsigned lt = (1u << lane) - 1u;
   const unsigned le = 0xffffffffu >> (31 - lane);
   if (gw >= gp.n_items) return;
@@ -261,7 +269,7 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
   // loads of the pass after it); one value set (reloaded once a pass's products are formed)
   ColRegs<E> nx;
   float vv[E];
-  load_cols<E>(a, gp.rs_bits, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, nx);
+  load_cols<E>(a, gp.rs_bits, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, nx, pol_ef);
   if (VALS) load_vals<E>(a, it.s, (int)(it.e - it.s), first_p0<E>(it) + E * lane, vv);
   for (;;) {
     const int64_t s = it.s;
@@ -271,15 +279,15 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
     if (lane == 0 && has_next) prefetch_item<VALS>(a, gp.items[nidx]);
     double dacc = 0.0;
     int nnzr = 0;
-    if (!chunk) {  // tile: non-empty rows -> list; empty rows finish here (y = 0)
+    if (!chunk) {  // tile: non-empty rows -> list (plan masks); empty rows finish here (y = 0)
       const int nr = it.r1 - it.r0;
+      const uint32_t *nzm = gp.tile_nz + 8 * (int64_t)it.t;
       for (int rb0 = 0; rb0 < nr; rb0 += 32) {
         const int r = rb0 + lane;
-        int d = 0;
-        if (r < nr) d = (int)(__ldg(a.row_ptr + it.r0 + r + 1) - __ldg(a.row_ptr + it.r0 + r));
-        const unsigned nz = __ballot_sync(0xffffffffu, r < nr && d > 0);
-        if (r < nr && d > 0) ws.nzrow[nnzr + __popc(nz & lt)] = (short)r;
-        if (r < nr && d == 0) dacc += epi(it.r0 + r, 0.0f);
+        const unsigned nz = ld_stream_pol(nzm + (rb0 >> 5), pol_ef);
+        const bool ne = (nz >> lane) & 1u;
+        if (ne) ws.nzrow[nnzr + __popc(nz & lt)] = (short)r;
+        if (r < nr && !ne) dacc += epi(it.r0 + r, 0.0f);
         nnzr += __popc(nz);
       }
     } else {  // a chunk is one row: its only start is offset 0
@@ -295,9 +303,9 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
       const int q0 = p0 + E * lane;
       const bool more = p0 + P < len;
       // (1) the next pass's columns (same item, or the next item's first pass)
-      if (more) load_cols<E>(a, gp.rs_bits, s, len, q0 + P, nx);
+      if (more) load_cols<E>(a, gp.rs_bits, s, len, q0 + P, nx, pol_ef);
       else if (has_next)
-        load_cols<E>(a, gp.rs_bits, ns, (int)(ne - ns), -(int)(ns & (E - 1)) + E * lane, nx);
+        load_cols<E>(a, gp.rs_bits, ns, (int)(ne - ns), -(int)(ns & (E - 1)) + E * lane, nx, pol_ef);
       // (2) my E row-start flags; entries outside the item gather the zero slot
       unsigned fl = (cur.fw >> (int)((s + q0) & 31)) & EM;
       if (!(p0 >= 0 && p0 + P <= len)) {  // edge pass of the item (warp-uniform)
@@ -316,7 +324,7 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
       float pr[E];
 #pragma unroll
       for (int j = 0; j < E; ++j) {
-        const float xv = gx((int32_t)cur.cv[j], xs_base, a.x);
+        const float xv = gx((int32_t)cur.cv[j], xs_base, a.x, pol);
         pr[j] = VALS ? vv[j] * xv : xv;
       }
       if (VALS) {  // the next pass's values
@@ -448,6 +456,7 @@ void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, con
   int64_t grid = ctx->num_sms;
   const int64_t need = (gp.n_items + NWARP - 1) / NWARP;
   if (grid > need) grid = need;
+  KScope ks(ctx, "k_gather");
   kern<<<(int)grid, NWARP * 32, smem, ctx->stream>>>(gp, a, epi);
   INL_CUDA(cudaGetLastError());
 }
@@ -480,6 +489,7 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
   gp.x_hot = (const float *)p->x_hot.p;
   gp.n_hot = (int)((p->n_hot + 3) & ~3);
   gp.rs_bits = (const uint32_t *)p->rs_bits.p;
+  gp.tile_nz = (const uint32_t *)p->tile_nz.p;
   gp.ticket = (unsigned long long *)p->ticket.p;
   // each launch advances the counter by exactly n_items (successful grabs + one failing
   // grab per active warp), so the next launch's base is known on the host: no reset

@@ -5,6 +5,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "inl.h"
 
@@ -13,11 +14,12 @@ namespace inl {
 constexpr int kTileRows = 256;  // max rows per SpMV/PR warp tile
 
 // One unit of work of the fused gather kernel (one warp): a tile (j < 0: rows [r0, r1),
-// all of degree <= t_warp, nonzeros [s, e)) or one chunk c of long row r0 (j = long-row
-// index, nonzeros [s, e), nch chunks, partial slots from pbase).
+// all of degree <= t_warp, nonzeros [s, e), tile index t into the plan's non-empty-row
+// masks) or one chunk c of long row r0 (j = long-row index, nonzeros [s, e), nch chunks,
+// partial slots from pbase).
 struct __align__(16) WorkItem {
   int64_t s, e;
-  int32_t r0, r1, j, c, nch, pbase, pad0, pad1;
+  int32_t r0, r1, j, c, nch, pbase, t, pad1;
 };
 
 struct Status {
@@ -70,6 +72,27 @@ Bins resolve_bins(const inl_bins *b);
 
 }  // namespace inl
 
+namespace inl {
+// Per-kernel launch timer (inl_ktimer_*): event pairs pending on the ctx stream, resolved
+// into (launches, ms) totals when read.
+struct KTimer {
+  struct Slot {
+    std::string name;
+    int64_t launches = 0;
+    double ms = 0.0;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending;
+  };
+  bool on = false;
+  std::vector<Slot> slots;
+  std::vector<cudaEvent_t> pool;
+  Slot &slot(const char *name);
+  cudaEvent_t ev();
+  void resolve();  // caller synchronized the stream
+  void clear();
+  ~KTimer();
+};
+}  // namespace inl
+
 struct inl_ctx_s {
   int device = 0;
   cudaStream_t stream = nullptr;
@@ -84,6 +107,7 @@ struct inl_ctx_s {
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
   bool closed = false;   // inl_ctx_destroy called; freed when the last plan goes
+  inl::KTimer ktimer;
 };
 
 struct inl_plan_s {
@@ -96,6 +120,7 @@ struct inl_plan_s {
   // tiles: rows [tile_lo[t], tile_hi[t]) with every row of degree <= t_warp
   int64_t n_tiles = 0;
   inl::DevBuf tiles;  // int2 {lo, hi}
+  inl::DevBuf tile_nz;  // uint32 [n_tiles * 8]: bit r of tile t = row lo_t + r is non-empty
   // long rows: degree > t_warp, cut into grid_chunk-sized chunks
   int64_t n_long = 0, n_chunks = 0;
   inl::DevBuf long_rows;    // int32 [n_long]
@@ -127,6 +152,24 @@ struct inl_plan_s {
 };
 
 namespace inl {
+// RAII bracket of one kernel launch for the kernel timer (no-op unless enabled).
+struct KScope {
+  inl_ctx ctx;
+  KTimer::Slot *sl = nullptr;
+  cudaEvent_t e0 = nullptr;
+  KScope(inl_ctx c, const char *name) : ctx(c) {
+    if (!c->ktimer.on) return;
+    sl = &c->ktimer.slot(name);
+    e0 = c->ktimer.ev();
+    cudaEventRecord(e0, c->stream);
+  }
+  ~KScope() {
+    if (!sl) return;
+    cudaEvent_t e1 = ctx->ktimer.ev();
+    cudaEventRecord(e1, ctx->stream);
+    sl->pending.emplace_back(e0, e1);
+  }
+};
 // plan.cu
 void build_plan(inl_plan p);
 // spmv.cu

@@ -85,7 +85,7 @@ __global__ void k_build_items(const int64_t *__restrict__ rp, const int2 *__rest
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
        i += (int64_t)gridDim.x * blockDim.x) {
     WorkItem w;
-    w.pad0 = w.pad1 = 0;
+    w.t = w.pad1 = 0;
     if (i < n_chunks) {
       const int2 ci = citems[i];
       const int32_t r = long_rows[ci.x];
@@ -105,11 +105,29 @@ __global__ void k_build_items(const int64_t *__restrict__ rp, const int2 *__rest
       w.r0 = t.x;
       w.r1 = t.y;
       w.j = -1;
+      w.t = (int32_t)(i - n_chunks);
       w.c = 0;
       w.nch = 0;
       w.pbase = 0;
     }
     out[i] = w;
+  }
+}
+
+// Non-empty-row masks of the tiles (one warp per tile): the gather kernel builds its
+// per-tile row lists from them instead of re-reading row_ptr.
+__global__ void k_tile_nz(const int64_t *__restrict__ rp, const int2 *__restrict__ tiles, int64_t n_tiles,
+                          uint32_t *__restrict__ nz) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t t = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; t < n_tiles;
+       t += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const int2 tl = tiles[t];
+    for (int rb = 0; rb < kTileRows; rb += 32) {
+      const int r = tl.x + rb + lane;
+      const bool ne = r < tl.y && rp[r + 1] > rp[r];
+      const unsigned m = __ballot_sync(0xffffffffu, ne);
+      if (lane == 0) nz[8 * t + rb / 32] = m;
+    }
   }
 }
 
@@ -308,6 +326,11 @@ void build_plan(inl_plan p) {
     k_build_items<<<grid_for(p->n_items, ctx->num_sms), 256, 0, st>>>(
         p->row_ptr, tiles, p->n_tiles, (const int2 *)p->chunk_items.p, (const int32_t *)p->long_rows.p,
         nch, (const int32_t *)p->chunk_base.p, p->n_chunks, b.grid_chunk, items);
+    INL_CUDA(cudaGetLastError());
+  }
+  if (p->n_tiles > 0) {
+    uint32_t *nz = (uint32_t *)p->tile_nz.get(sizeof(uint32_t) * 8 * p->n_tiles);
+    k_tile_nz<<<grid_for(p->n_tiles * 32, ctx->num_sms), 256, 0, st>>>(p->row_ptr, tiles, p->n_tiles, nz);
     INL_CUDA(cudaGetLastError());
   }
   p->dpart.get(sizeof(double) * (p->n_items + 1));

@@ -27,6 +27,7 @@ __device__ __forceinline__ uint32_t ld_stream_32(const void *p) {
   return r;
 }
 
+
 // Streaming 32-bit load with an L2 eviction policy (createpolicy), no L1 allocation.
 __device__ __forceinline__ uint32_t ld_stream_pol(const void *p, uint64_t pol) {
   uint32_t r;

@@ -30,6 +30,7 @@ void spmv_thread_only(inl_ctx ctx, const inl_csr &A, const float *val, const flo
   GatherArgs a{A.row_ptr, A.col_idx, val, x, A.nnz, A.n_rows, 0, 0, 0, 0, false};
   int64_t g = (A.n_rows + 255) / 256;
   if (g > (int64_t)ctx->num_sms * 32) g = (int64_t)ctx->num_sms * 32;
+  KScope ks(ctx, "k_gather_thread_only");
   k_gather_thread_only<<<(int)g, 256, 0, ctx->stream>>>(A.n_rows, a, SpmvEpi{y});
   INL_CUDA(cudaGetLastError());
 }

@@ -84,9 +84,12 @@ def lib() -> C.CDLL:
         L.inl_pagerank.argtypes = [vp, C.POINTER(CsrT), vp, C.c_float, i32, vp, vp]
         L.inl_sssp.argtypes = [vp, C.POINTER(CsrT), vp, i64, vp, C.POINTER(StatsT), vp]
         L.inl_bfs.argtypes = [vp, C.POINTER(CsrT), i64, vp, C.POINTER(StatsT), vp]
+        L.inl_ktimer_enable.argtypes = [vp, i32]
+        L.inl_ktimer_read.argtypes = [vp, C.c_char_p, C.POINTER(i64), C.POINTER(C.c_double)]
         for f in ("inl_ctx_create", "inl_ctx_set_stream", "inl_ctx_destroy", "inl_partition_rows",
                   "inl_nccl_unique_id", "inl_comm_init", "inl_plan_create", "inl_plan_get_info",
-                  "inl_plan_destroy", "inl_csr_validate", "inl_spmv", "inl_pagerank", "inl_sssp", "inl_bfs"):
+                  "inl_plan_destroy", "inl_csr_validate", "inl_spmv", "inl_pagerank", "inl_sssp", "inl_bfs",
+                  "inl_ktimer_enable", "inl_ktimer_read"):
             getattr(L, f).restype = C.c_int
         _lib = L
     return _lib
@@ -167,6 +170,16 @@ class Ctx:
         _check(lib().inl_comm_init(self.handle, uid.ctypes.data, nranks, rank), self)
         self.nranks, self.rank = nranks, rank
 
+    def ktimer_enable(self, on: bool = True) -> None:
+        """Bracket the main kernels' launches with CUDA events (measurement only)."""
+        _check(lib().inl_ktimer_enable(self.handle, 1 if on else 0), self)
+
+    def ktimer_read(self, kernel: str) -> tuple[int, float]:
+        """(launches, summed device ms) of `kernel` since ktimer_enable (syncs the stream)."""
+        n, ms = C.c_int64(), C.c_double()
+        _check(lib().inl_ktimer_read(self.handle, kernel.encode(), C.byref(n), C.byref(ms)), self)
+        return int(n.value), float(ms.value)
+
     def close(self) -> None:
         if getattr(self, "handle", None):
             lib().inl_ctx_destroy(self.handle)
@@ -222,6 +235,16 @@ class Plan:
         d = {f: getattr(i, f) for f, _ in PlanInfoT._fields_ if f != "bins"}
         d["bins"] = {f: getattr(i.bins, f) for f, _ in BinsT._fields_}
         return d
+
+    def ktimer_enable(self, on: bool = True) -> None:
+        """Bracket the main kernels' launches with CUDA events (measurement only)."""
+        _check(lib().inl_ktimer_enable(self.handle, 1 if on else 0), self)
+
+    def ktimer_read(self, kernel: str) -> tuple[int, float]:
+        """(launches, summed device ms) of `kernel` since ktimer_enable (syncs the stream)."""
+        n, ms = C.c_int64(), C.c_double()
+        _check(lib().inl_ktimer_read(self.handle, kernel.encode(), C.byref(n), C.byref(ms)), self)
+        return int(n.value), float(ms.value)
 
     def close(self) -> None:
         if getattr(self, "handle", None):
