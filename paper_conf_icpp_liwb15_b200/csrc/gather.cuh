@@ -90,7 +90,7 @@ struct PrEpi {
   __device__ __forceinline__ double operator()(int64_t r, float s) const {
     const int64_t v = row_begin + r;
     const float pr = fmaf(damping, s, base);
-    const int od = __ldg(out_degree + v);
+    const int od = __ldg(out_degree + v);  // L1-cached: neighbouring rows share lines
     if (od > 0) c_next[__ldg(cidx + v)] = pr / (float)od;
     if (rank_out) rank_out[v] = pr;
     return od == 0 ? (double)pr : 0.0;
