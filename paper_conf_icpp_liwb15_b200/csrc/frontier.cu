@@ -43,6 +43,27 @@ __device__ __forceinline__ void push(int32_t *q, int *cnt, int32_t v) {
   q[pos] = v;
 }
 
+// Warp-aggregated enqueue of the slots of m (bit j: v[j]) — one counter atomic per warp.
+// All 32 lanes must call it (warp-uniform control flow).
+template <int K>
+__device__ __forceinline__ void push_batch(int32_t *q, int *cnt, const int32_t (&v)[K], unsigned m) {
+  if (!__any_sync(0xffffffffu, m != 0u)) return;
+  const int lane = threadIdx.x & 31;
+  const int c = __popc(m);
+  int incl = c;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int t = __shfl_up_sync(0xffffffffu, incl, d);
+    if (lane >= d) incl += t;
+  }
+  int base = 0;
+  if (lane == 31) base = atomicAdd(cnt, incl);
+  int pos = __shfl_sync(0xffffffffu, base, 31) + incl - c;
+#pragma unroll
+  for (int j = 0; j < K; ++j)
+    if ((m >> j) & 1u) q[pos++] = v[j];
+}
+
 struct SsspOp {
   uint32_t *dist;       // [n_global (+1 flag word on P > 1)]
   const uint32_t *w;    // [nnz]
@@ -59,24 +80,60 @@ struct SsspOp {
   __device__ __forceinline__ uint32_t load(int32_t u) const {
     return *(volatile uint32_t *)(dist + row_begin + u);
   }
-  __device__ __forceinline__ void edge(uint32_t du, int64_t k, int32_t v, int32_t *q, int *cnt) const {
-    const uint32_t nd = du + __ldg(w + k);
-    if (nd < dist[v]) {
-      const uint32_t old = atomicMin(dist + v, nd);
-      if (nd < old) {
-        if (enqueue) {
-          if (nd >= thr) {
-            const uint32_t bit = 1u << (v & 31);
-            if (!(atomicOr(infar + (v >> 5), bit) & bit)) push(far, far_count, v);
-          } else {
-            const uint32_t bit = 1u << (v & 31);
-            if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, cnt, v);
-          }
+  __device__ __forceinline__ void improve(int32_t v, uint32_t nd, int32_t *q, int *cnt) const {
+    const uint32_t old = atomicMin(dist + v, nd);
+    if (nd < old) {
+      if (enqueue) {
+        const uint32_t bit = 1u << (v & 31);
+        if (nd >= thr) {
+          if (!(atomicOr(infar + (v >> 5), bit) & bit)) push(far, far_count, v);
         } else {
-          *flag = 0u;
+          if (!(atomicOr(inq + (v >> 5), bit) & bit)) push(q, cnt, v);
         }
+      } else {
+        *flag = 0u;
       }
     }
+  }
+  __device__ __forceinline__ void edge(uint32_t du, int64_t k, int32_t v, int32_t *q, int *cnt) const {
+    const uint32_t nd = du + __ldg(w + k);
+    if (nd < dist[v]) improve(v, nd, q, cnt);
+  }
+  // K edges per lane at once, every stage issued back to back so the latencies overlap
+  // (memory-level parallelism K): weight loads, dist gathers, atomicMin of the candidate
+  // improvements, claim bits of the improved vertices, one warp-aggregated enqueue.
+  // Out-of-range slots have in[j] = false.  All 32 lanes must call it.
+  template <int K>
+  __device__ __forceinline__ void edges(const uint32_t (&du)[K], const int64_t (&kk)[K], const int32_t (&vv)[K],
+                                        const bool (&in)[K], int32_t *q, int *cnt) const {
+    uint32_t nd[K], dv[K], old[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j) nd[j] = in[j] ? du[j] + ld_stream_pol(w + kk[j], pol_stream) : 0xFFFFFFFFu;
+#pragma unroll
+    for (int j = 0; j < K; ++j) dv[j] = in[j] ? dist[vv[j]] : 0u;
+#pragma unroll
+    for (int j = 0; j < K; ++j) old[j] = nd[j] < dv[j] ? atomicMin(dist + vv[j], nd[j]) : 0u;
+    unsigned imp = 0u;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (nd[j] < dv[j] && nd[j] < old[j]) imp |= 1u << j;
+    if (!enqueue) {
+      if (imp) *flag = 0u;
+      return;
+    }
+    uint32_t ob[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      ob[j] = (imp >> j) & 1u ? atomicOr((nd[j] >= thr ? infar : inq) + (vv[j] >> 5), 1u << (vv[j] & 31)) : 0u;
+    unsigned nearm = 0u, farm = 0u;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (((imp >> j) & 1u) && !((ob[j] >> (vv[j] & 31)) & 1u)) {
+        if (nd[j] >= thr) farm |= 1u << j;
+        else nearm |= 1u << j;
+      }
+    push_batch(q, cnt, vv, nearm);
+    push_batch(far, far_count, vv, farm);
   }
 };
 
@@ -89,20 +146,52 @@ struct BfsOp {
   bool enqueue;      // !DIST
   uint64_t pol_stream;
   __device__ __forceinline__ uint32_t load(int32_t) const { return 0u; }
+  __device__ __forceinline__ void visit(int32_t v, int32_t *q, int *cnt) const {
+    if (enqueue) {
+      const uint32_t bit = 1u << (v & 31);
+      const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
+      if (!(old & bit)) {
+        level[v] = L + 1;
+        push(q, cnt, v);
+      }
+    } else {
+      next[v] = 1;
+      next[n] = 1;
+    }
+  }
   __device__ __forceinline__ void edge(uint32_t, int64_t, int32_t v, int32_t *q, int *cnt) const {
     const uint32_t bit = 1u << (v & 31);
-    if (!(bitmap[v >> 5] & bit)) {
-      if (enqueue) {
-        const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
-        if (!(old & bit)) {
-          level[v] = L + 1;
-          push(q, cnt, v);
-        }
-      } else {
-        next[v] = 1;
-        next[n] = 1;
-      }
+    if (!(bitmap[v >> 5] & bit)) visit(v, q, cnt);
+  }
+  // K edges per lane at once (see SsspOp::edges); all 32 lanes must call it.
+  template <int K>
+  __device__ __forceinline__ void edges(const uint32_t (&)[K], const int64_t (&)[K], const int32_t (&vv)[K],
+                                        const bool (&in)[K], int32_t *q, int *cnt) const {
+    uint32_t bw[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j) bw[j] = in[j] ? bitmap[vv[j] >> 5] : 0xFFFFFFFFu;
+    unsigned cand = 0u;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (!((bw[j] >> (vv[j] & 31)) & 1u)) cand |= 1u << j;
+    if (!enqueue) {
+#pragma unroll
+      for (int j = 0; j < K; ++j)
+        if ((cand >> j) & 1u) next[vv[j]] = 1;
+      if (cand) next[n] = 1;
+      return;
     }
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      bw[j] = (cand >> j) & 1u ? atomicOr(bitmap + (vv[j] >> 5), 1u << (vv[j] & 31)) : 0xFFFFFFFFu;
+    unsigned won = 0u;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (((cand >> j) & 1u) && !((bw[j] >> (vv[j] & 31)) & 1u)) {
+        won |= 1u << j;
+        level[vv[j]] = L + 1;
+      }
+    push_batch(q, cnt, vv, won);
   }
 };
 
@@ -232,34 +321,33 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
   const int nruns = tot.x, total = tot.y;
   if (tid == 0) off_s[nruns] = total;
   __syncthreads();
-  for (int w0 = 0; w0 < total; w0 += NT * kEdgesPerThread) {
-    int e = w0 + tid * kEdgesPerThread;
-    if (e >= total) continue;
-    int lo = 0, hi = nruns;  // last run with off_s[run] <= e
+  // each warp takes 32*K consecutive edges of the window; lane l takes edges l, l+32, ...
+  // (every load instruction of the warp reads 32 consecutive edges: coalesced)
+  for (int w0 = warp * 32 * kEdgesPerThread; w0 < total; w0 += NT * kEdgesPerThread) {
+    const int e0 = w0 + lane;
+    int lo = 0, hi = nruns;  // last run with off_s[run] <= e0
+    const int es = e0 < total ? e0 : total - 1;
     while (hi - lo > 1) {
       const int mid = (lo + hi) >> 1;
-      if (off_s[mid] <= e) lo = mid; else hi = mid;
+      if (off_s[mid] <= es) lo = mid; else hi = mid;
     }
-    int run = lo, rend = off_s[lo + 1];
+    int run = lo;
     int64_t kk[kEdgesPerThread];
     uint32_t du[kEdgesPerThread];
     int32_t vv[kEdgesPerThread];
     bool in[kEdgesPerThread];
 #pragma unroll
     for (int j = 0; j < kEdgesPerThread; ++j) {
-      in[j] = e + j < total;
-      if (in[j] && e + j >= rend) {  // runs are non-empty: one step reaches the next run
-        ++run;
-        rend = off_s[run + 1];
-      }
-      kk[j] = rs_s[run] + (e + j - off_s[run]);
+      const int e = e0 + 32 * j;
+      in[j] = e < total;
+      if (in[j])
+        while (off_s[run + 1] <= e) ++run;  // runs are non-empty: forward walk
+      kk[j] = rs_s[run] + (e - off_s[run]);
       du[j] = su_s[run];
     }
 #pragma unroll
-    for (int j = 0; j < kEdgesPerThread; ++j) vv[j] = in[j] ? __ldg(a.col + kk[j]) : 0;
-#pragma unroll
-    for (int j = 0; j < kEdgesPerThread; ++j)
-      if (in[j]) op.edge(du[j], kk[j], vv[j], a.Fout, a.fcount);
+    for (int j = 0; j < kEdgesPerThread; ++j) vv[j] = in[j] ? (int32_t)ld_stream_pol(a.col + kk[j], op.pol_stream) : 0;
+    op.edges(du, kk, vv, in, a.Fout, a.fcount);
   }
   for (int o = 16; o > 0; o >>= 1) mydeg += __shfl_xor_sync(0xffffffffu, mydeg, o);
   if (lane == 0) red[warp] = mydeg;
@@ -283,18 +371,20 @@ __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
     const int64_t ks = rs + (int64_t)g.y * a.chunk;
     const int64_t ke = min(ks + (int64_t)a.chunk, re);
     const uint32_t su = op.load(g.x);
-    for (int64_t k0 = ks + threadIdx.x; k0 < ke; k0 += NT * kEdgesPerThread) {
+    for (int64_t kb = ks; kb < ke; kb += NT * kEdgesPerThread) {  // block-uniform trip count
+      const int64_t k0 = kb + threadIdx.x;
       int32_t vv[kEdgesPerThread];
+      int64_t kk[kEdgesPerThread];
+      uint32_t du[kEdgesPerThread];
+      bool in[kEdgesPerThread];
 #pragma unroll
       for (int j = 0; j < kEdgesPerThread; ++j) {
-        const int64_t k = k0 + (int64_t)j * NT;
-        vv[j] = k < ke ? (int32_t)ld_stream_pol(a.col + k, op.pol_stream) : 0;
+        kk[j] = k0 + (int64_t)j * NT;
+        in[j] = kk[j] < ke;
+        du[j] = su;
+        vv[j] = in[j] ? (int32_t)ld_stream_pol(a.col + kk[j], op.pol_stream) : 0;
       }
-#pragma unroll
-      for (int j = 0; j < kEdgesPerThread; ++j) {
-        const int64_t k = k0 + (int64_t)j * NT;
-        if (k < ke) op.edge(su, k, vv[j], a.Fout, a.fcount);
-      }
+      op.edges(du, kk, vv, in, a.Fout, a.fcount);
     }
   }
 }
