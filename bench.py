@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--edge-factor", type=int, default=16)
     ap.add_argument("--bins", type=str, default="", help="t_thread,t_warp,t_block,grid_chunk,cta")
     ap.add_argument("--thread-only", action="store_true", help="paper baseline T1 (no load balancing)")
+    ap.add_argument("--colblock", action="store_true", help="long rows column-blocked (INL_BINS_COLBLOCK)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--iterations", type=int, default=20, help="PageRank iterations")
@@ -186,7 +187,8 @@ def run_inl(a):
     g = W["g"]
     A = inl.Csr(g["row_ptr"], g["col_idx"], g["n_global"], g["row_begin"])
     bargs = [int(v) for v in a.bins.split(",")] if a.bins else []
-    bb = inl.bins(*bargs, flags=inl.BINS_THREAD_ONLY if a.thread_only else 0)
+    bb = inl.bins(*bargs, flags=(inl.BINS_THREAD_ONLY if a.thread_only else 0) |
+                  (inl.BINS_COLBLOCK if a.colblock else 0))
     t0 = time.perf_counter()
     plan = inl.Plan(ctx, A, bb)
     torch.cuda.synchronize()
@@ -201,13 +203,14 @@ def run_inl(a):
         step = lambda: inl.spmv(ctx, A, W["val"], W["x"], y, plan)  # noqa: E731
         units_local = nnz_local
         bytes_local = spmv_bytes(nnz_local, A.n_rows, A.n_global)
-        launches_per_step = 2 if info["bins"]["flags"] == 0 else 1  # k_build_xhot + k_gather
+        # k_build_xhot + k_gather (+ k_cb + k_cb_combine when rows are column-blocked)
+        launches_per_step = (1 if a.thread_only else 2) + (2 if info["cb_rows"] > 0 else 0)
     elif a.op == "pagerank":
         r = torch.empty(A.n_global, device="cuda")
         step = lambda: inl.pagerank(ctx, A, g["out_degree"], r, 0.85, a.iterations, plan)  # noqa: E731
         units_local = nnz_local * a.iterations
         bytes_local = pagerank_bytes_per_iter(nnz_local, A.n_rows, A.n_global) * a.iterations
-        launches_per_step = 3 + 4 * a.iterations  # init; per iteration xhot + gather + dsum + base
+        launches_per_step = None  # counted by the library's kernel timer below
     else:
         # seeded sources of degree > 0 (+ the max-degree vertex); under torchrun rank 0 picks
         # them from its row block (global ids: its row_begin is 0) and broadcasts them
@@ -240,7 +243,8 @@ def run_inl(a):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     reached = []
     # the dominant kernel(s), timed live by the library with events on its own stream
-    kernels = ["k_gather"] if a.op in ("spmv", "pagerank") else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up"]
+    kernels = (["k_gather", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
+               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
     ctx.ktimer_enable(True)
@@ -254,11 +258,19 @@ def run_inl(a):
         ev1.record(stream)
         torch.cuda.synchronize()
     ms = ev0.elapsed_time(ev1)
-    k_launches, k_ms = 0, 0.0
+    k_launches, k_ms, k_used, k_each = 0, 0.0, [], {}
     for kn in kernels:
         nl, kms = ctx.ktimer_read(kn)
         k_launches += nl
         k_ms += kms
+        if nl:
+            k_used.append(kn)
+            k_each[kn] = {"launches": nl, "ms_per_launch": round(kms / nl, 5)}
+    if a.op == "pagerank":
+        # per step: init + base0; per iteration: x_hot + gather (+ k_cb + combine); between
+        # iterations: dangling sum + base
+        cb_on = "k_cb" in k_used
+        launches_per_step = 2 + a.iterations * (4 if cb_on else 2) + (a.iterations - 1) * 2
     ctx.ktimer_enable(False)
     if world > 1:
         t = torch.tensor([ms], device="cuda")
@@ -322,7 +334,7 @@ def run_inl(a):
         out["roofline"] = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak, "unit": "GB/s",
                            "frac": round(frac, 4), "peak_source": peak_src,
                            "frac_of_8TBs": round(achieved_gbs / 8000.0, 4),
-                           "kernel": "+".join(kernels),
+                           "kernel": "+".join(k_used or kernels), "kernels": k_each,
                            "kernel_launches": k_launches, "kernel_ms_per_launch": round(k_ms / max(k_launches, 1), 5),
                            "kernel_share_of_step": round(k_ms / ms, 4),
                            "alg_bytes_per_step_per_gpu": int(bytes_total / world / a.steps),

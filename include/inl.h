@@ -69,8 +69,12 @@ typedef struct {
  * Ties go to the lower bin (reading R6 of DESIGN.md: "f(i) greater than lbTHRES
  * is processed block-mapped", P11@1197).  t_thread = -1 means 0 (no thread bin).
  * flags: INL_BINS_THREAD_ONLY runs the paper's baseline (thread-mapped outer loop,
- * no load balancing, P5@14490). */
-enum { INL_BINS_THREAD_ONLY = 1 };
+ * no load balancing, P5@14490).  INL_BINS_COLBLOCK (opt-in; measured slower at the
+ * bench configs) processes SpMV/PR rows of degree > max(t_warp,
+ * 4 * column blocks) column-blocked: a CTA holds one block of x in shared memory and
+ * sums the row's entries in that block (one partial per (row, block) run, combined in
+ * block order). */
+enum { INL_BINS_THREAD_ONLY = 1, INL_BINS_COLBLOCK = 2 };
 typedef struct {
   int32_t t_thread;    /* default 8 */
   int32_t t_warp;      /* default 128, in [16, 4096] (SpMV/PR warp tiles hold < 2*t_warp nnz) */
@@ -93,6 +97,11 @@ typedef struct {
   int64_t nnz_thread, nnz_warp, nnz_block, nnz_grid;
   int64_t n_grid_chunks;  /* CTAs of the grid/long-row kernel */
   inl_bins bins;          /* thresholds in effect */
+  int64_t cb_rows;        /* SpMV rows processed column-blocked (0: none) */
+  int64_t cb_runs;        /* their (row, column block) runs = partial sums */
+  int64_t cb_nnz;         /* their nonzeros */
+  int64_t cb_width;       /* column-block width K (x floats held in shared memory) */
+  int64_t cb_threshold;   /* rows of degree > cb_threshold are column-blocked */
 } inl_plan_info;
 
 const char *inl_version(void);

@@ -34,6 +34,7 @@
 #pragma once
 #include <cuda/atomic>
 
+#include "colblock.cuh"
 #include "inl_internal.cuh"
 #include "ptx.cuh"
 
@@ -473,35 +474,48 @@ inline int gather_entries_per_lane() {
 // Host-side launcher for one full gather (tiles + long-row chunks) on a plan; x is the
 // dense vector (n_global) whose hot part is copied to the plan's x_hot first.
 // col_over / hot_over: a column space other than the plan's (PageRank's compacted one).
+// cb: the column-blocked bin of that column space (its rows leave the gather's items and
+// are summed by k_cb + k_cb_combine; their dangling values go to dpart[n_items + j]).
 template <bool VALS, class Epi>
 void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart,
-                   const int32_t *col_over = nullptr, const int32_t *hot_over = nullptr) {
+                   const int32_t *col_over = nullptr, const int32_t *hot_over = nullptr,
+                   const CbPlan *cb = nullptr) {
   if (p->n_items == 0) return;
+  const bool use_cb = cb && cb->active;
+  const int64_t n_items = use_cb ? cb->n_items : p->n_items;
   GatherArgs a = a_in;
   if (col_over) a.col_idx = col_over;
   else if (p->n_hot > 0) a.col_idx = (const int32_t *)p->pcol.p;  // hot columns remapped
-  GatherPlan gp;
-  gp.items = (const WorkItem *)p->items.p;
-  gp.n_items = (int)p->n_items;
-  gp.partials = (float *)p->partials.p;
-  gp.tickets = (int *)p->tickets.p;
-  gp.dpart = dpart;
-  gp.x_hot = (const float *)p->x_hot.p;
-  gp.n_hot = (int)((p->n_hot + 3) & ~3);
-  gp.rs_bits = (const uint32_t *)p->rs_bits.p;
-  gp.tile_nz = (const uint32_t *)p->tile_nz.p;
-  gp.ticket = (unsigned long long *)p->ticket.p;
-  // each launch advances the counter by exactly n_items (successful grabs + one failing
-  // grab per active warp), so the next launch's base is known on the host: no reset
-  gp.base = p->ticket_base;
-  p->ticket_base += (unsigned long long)p->n_items;
-  build_xhot(ctx, p, a.x, hot_over);
-  a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
-  static int w24 = -1;
-  if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;
-  if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi);
-  else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi);
-  else launch_gather_t<8, VALS>(ctx, gp, a, epi);
+  if (n_items > 0) {
+    GatherPlan gp;
+    gp.items = (const WorkItem *)(use_cb ? cb->items.p : p->items.p);
+    gp.n_items = (int)n_items;
+    gp.partials = (float *)p->partials.p;
+    gp.tickets = (int *)p->tickets.p;
+    gp.dpart = dpart;
+    gp.x_hot = (const float *)p->x_hot.p;
+    gp.n_hot = (int)((p->n_hot + 3) & ~3);
+    gp.rs_bits = (const uint32_t *)p->rs_bits.p;
+    gp.tile_nz = (const uint32_t *)p->tile_nz.p;
+    gp.ticket = (unsigned long long *)p->ticket.p;
+    // each launch advances the counter by exactly n_items (successful grabs + one failing
+    // grab per active warp), so the next launch's base is known on the host: no reset
+    gp.base = p->ticket_base;
+    p->ticket_base += (unsigned long long)n_items;
+    build_xhot(ctx, p, a.x, hot_over);
+    a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
+    static int w24 = -1;
+    if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;
+    if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi);
+    else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi);
+    else launch_gather_t<8, VALS>(ctx, gp, a, epi);
+  }
+  if (use_cb) launch_cb<VALS>(ctx, *cb, a_in.val, a_in.x, epi, dpart ? dpart + n_items : nullptr);
+}
+
+// number of dangling partials launch_gather writes
+inline int64_t gather_dpart_count(inl_plan p, const CbPlan *cb) {
+  return cb && cb->active ? cb->n_items + cb->n_rows : p->n_items;
 }
 
 }  // namespace inl

@@ -70,6 +70,38 @@ struct Bins {
 };
 Bins resolve_bins(const inl_bins *b);
 
+// One (column block, row) run of a column-blocked row (colblock.cu): entries
+// [cs, cs + len) of the CSR, whose columns all lie in one column block; their local
+// column offsets are cbcol[cb, cb + len).  j = index of the row in CbPlan::rows.
+struct __align__(8) CbPair {
+  int64_t cs, cb;
+  int32_t len, j;
+};
+
+// Column-blocked deferred bin: rows of degree > t_cb are split by column
+// block (K consecutive columns = one shared-memory copy of x); a CTA loads one block of x
+// and sums every run of that block into a per-run partial; a combine kernel adds each
+// row's partials in block order.  Built per column space (SpMV: the CSR's; PageRank: the
+// compacted contribution space).
+struct CbPlan {
+  bool active = false;
+  int K = 0;                // column-block width (x slots in shared memory)
+  int64_t ncols = 0, nblocks = 0;
+  int32_t t_cb = 0;         // rows of degree > t_cb are column-blocked
+  int64_t n_rows = 0, n_pairs = 0, n_entries = 0;
+  int grid = 0;             // CTAs of k_cb (entry ranges in cta_lo)
+  DevBuf rows;              // int32 [n_rows] local row ids
+  DevBuf rp_base;           // int64 [n_rows + 1] first run (row order) of each row
+  DevBuf pos_of;            // int64 [n_pairs] position of run q (row order) in `pairs`
+  DevBuf pairs;             // CbPair [n_pairs] sorted by (block, length desc, row)
+  DevBuf blk_first;         // int64 [nblocks + 1] first pair of each block
+  DevBuf cta_lo;            // int64 [grid + 1] first pair of each CTA (equal entry shares)
+  DevBuf cbcol;             // uint16 [n_entries] column offsets within the block
+  DevBuf partials;          // float [n_pairs]
+  int64_t n_items = 0;      // gather work items without the column-blocked rows
+  DevBuf items;             // WorkItem [n_items]
+};
+
 }  // namespace inl
 
 namespace inl {
@@ -149,6 +181,8 @@ struct inl_plan_s {
   inl::DevBuf pr_cidx;         // int32 [n_global]: exchange-space index, -1 if dangling
   inl::DevBuf pr_col;          // int32 [nnz]: gather columns in the compact space (hot kept)
   inl::DevBuf pr_hot;          // int32 [n_hot]: hot slots in the compact space
+  // column-blocked long rows: SpMV (the CSR's column space) and PageRank (compact space)
+  inl::CbPlan cb, pr_cb;
 };
 
 namespace inl {
@@ -183,6 +217,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
               uint32_t *dist, inl_stats *st);
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
              inl_stats *st);
+// colblock.cu: builds `cb` for the column space `cols` (raw ids in [0, ncols), CSR order)
+void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool sort_rows = false);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);
 }  // namespace inl

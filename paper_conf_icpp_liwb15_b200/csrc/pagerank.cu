@@ -3,9 +3,12 @@
 // rows; epilogue computes PR', the next contribution and the dangling partials)
 // + one single-CTA fixed-order reduction of the dangling partials.  On P > 1
 // ranks the contribution slice and the rank's dangling sum are allgathered.
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include <algorithm>
+#include <cstdlib>
+#include <string>
 #include <vector>
 
 #include "comm.h"
@@ -83,6 +86,29 @@ __global__ void k_cidx(const int32_t *__restrict__ od, const int32_t *__restrict
   }
 }
 
+// degree order: key = (rank block q, ~out_degree) so that, after a stable sort, block q's
+// pages with out-links come first in descending out-degree (ties by id), dangling last
+__global__ void k_deg_keys(const int32_t *__restrict__ od, int64_t n, int64_t B, uint64_t *__restrict__ key,
+                           int32_t *__restrict__ ids) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    key[v] = ((uint64_t)(v / B) << 32) | (uint64_t)(~(uint32_t)max(od[v], 0));
+    ids[v] = (int32_t)v;
+  }
+}
+
+// slot of the i-th vertex of the sorted order within its block (blocks are contiguous runs
+// of B positions in the sorted order)
+__global__ void k_cidx_sorted(const int32_t *__restrict__ od, const int32_t *__restrict__ ids, int64_t n,
+                              int64_t B, int64_t Bc, int32_t *__restrict__ cidx) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = ids[i];
+    const int64_t q = v / B;
+    cidx[v] = od[v] > 0 ? (int32_t)(q * Bc + (i - q * B)) : -1;
+  }
+}
+
 // gather columns in the compact space (hot slots kept); a column without out-links
 // (inconsistent input) reads the zero slot
 __global__ void k_remap_cols(const int32_t *__restrict__ col, int64_t nnz, const int32_t *__restrict__ cidx,
@@ -117,6 +143,9 @@ int grid_for(int64_t n, int sms) {
 
 // Compact (exchange-space) numbering of the pages with out-links, the gather columns in
 // that space, and the slots per rank block.  Cached in the plan per out_degree array.
+// Inside a rank block the slots follow descending out-degree (= how often a page's
+// contribution is gathered), so the frequently read contributions share cache lines
+// and stay L2-resident; INL_PR_ORDER=vertex keeps vertex order (measurement switch).
 static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, int P) {
   if (p->pr_od == od) return;
   cudaStream_t st = ctx->stream;
@@ -137,7 +166,27 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
   for (int q = 0; q < P; ++q) bc = std::max<int64_t>(bc, (int64_t)at[q + 1] - at[q]);
   p->pr_bc = bc;
   int32_t *cidx = (int32_t *)p->pr_cidx.get(sizeof(int32_t) * (n > 0 ? n : 1));
-  k_cidx<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, pos, n, B, bc, cidx);
+  static int vorder = -1;
+  if (vorder < 0) {
+    const char *e = getenv("INL_PR_ORDER");
+    vorder = e && std::string(e) == "vertex";
+  }
+  if (vorder || n <= 1) {
+    k_cidx<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, pos, n, B, bc, cidx);
+  } else {
+    uint64_t *k0 = (uint64_t *)ctx->s_a.get(sizeof(uint64_t) * n);
+    uint64_t *k1 = (uint64_t *)ctx->s_b.get(sizeof(uint64_t) * n);
+    int32_t *i0 = flags, *i1 = pos;  // the scan results are no longer needed
+    k_deg_keys<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, n, B, k0, i0);
+    int end_bit = 32;
+    while (end_bit < 64 && ((uint64_t)(P - 1) >> (end_bit - 32))) ++end_bit;
+    cub::DoubleBuffer<uint64_t> kb(k0, k1);
+    cub::DoubleBuffer<int32_t> vb(i0, i1);
+    size_t sneed = 0;
+    INL_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, sneed, kb, vb, n, 0, end_bit, st));
+    INL_CUDA(cub::DeviceRadixSort::SortPairs(ctx->s_tmp.get(sneed), sneed, kb, vb, n, 0, end_bit, st));
+    k_cidx_sorted<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, vb.Current(), n, B, bc, cidx);
+  }
   const int32_t zero_slot = (int32_t)(bc * P);
   const int32_t *src = p->n_hot > 0 ? (const int32_t *)p->pcol.p : p->col_idx;
   int32_t *pc = (int32_t *)p->pr_col.get(sizeof(int32_t) * (p->nnz > 0 ? p->nnz : 1));
@@ -149,6 +198,14 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
                                                                  cidx, zero_slot, ph);
   }
   INL_CUDA(cudaGetLastError());
+  {  // column-blocked bin in the compact space (raw compact columns, no hot tags)
+    DevBuf raw;
+    int32_t *rc = (int32_t *)raw.get(sizeof(int32_t) * (p->nnz > 0 ? p->nnz : 1));
+    if (p->nnz > 0)
+      k_remap_cols<<<grid_for(p->nnz, ctx->num_sms), 256, 0, st>>>(p->col_idx, p->nnz, cidx, zero_slot, rc);
+    INL_CUDA(cudaGetLastError());
+    cb_build(p, p->pr_cb, rc, bc * P + 1, /*sort_rows=*/!vorder);
+  }
   p->pr_od = od;
 }
 
@@ -187,7 +244,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
   k_pr_base0<<<1, 1, 0, st>>>(ndang, n, (double)damping, base);
   INL_CUDA(cudaGetLastError());
 
-  const int64_t m = p->n_items;
+  const int64_t m = gather_dpart_count(p, &p->pr_cb);
   double *dpart = (double *)p->dpart.p;
   for (int t = 0; t < iters; ++t) {
     const bool last = t + 1 == iters;
@@ -196,7 +253,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
     PrEpi epi{out_degree, c_next, cidx, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
               p->row_begin, 0.0f};
     launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p,
-                         p->n_hot > 0 ? (const int32_t *)p->pr_hot.p : nullptr);
+                         p->n_hot > 0 ? (const int32_t *)p->pr_hot.p : nullptr, &p->pr_cb);
     if (!last) {
       k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
       INL_CUDA(cudaGetLastError());

@@ -342,6 +342,8 @@ void build_plan(inl_plan p) {
     INL_CUDA(cudaGetLastError());
   }
   build_hot_remap(p);
+  cb_build(p, p->cb, p->col_idx, p->n_global);
+  p->pr_cb.active = false;
   INL_CUDA(cudaMemsetAsync(p->ticket.get(16), 0, 16, st));
   p->ticket_base = 0;
   p->info.n_tiles = p->n_tiles;
@@ -354,6 +356,11 @@ void build_plan(inl_plan p) {
   p->info.nnz_block = (int64_t)h_st[6];
   p->info.nnz_grid = (int64_t)h_st[7];
   p->info.n_grid_chunks = p->n_chunks;
+  p->info.cb_rows = p->cb.active ? p->cb.n_rows : 0;
+  p->info.cb_runs = p->cb.active ? p->cb.n_pairs : 0;
+  p->info.cb_nnz = p->cb.active ? p->cb.n_entries : 0;
+  p->info.cb_width = p->cb.active ? p->cb.K : 0;
+  p->info.cb_threshold = p->cb.active ? p->cb.t_cb : 0;
 }
 
 }  // namespace inl

@@ -22,7 +22,7 @@ void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols
 void spmv_run(inl_ctx ctx, inl_plan p, const float *val, const float *x, float *y) {
   GatherArgs a{p->row_ptr, p->col_idx, val, x, p->nnz, p->n_rows,
                p->bins.t_thread, p->bins.t_warp, p->bins.t_block, p->bins.grid_chunk, false};
-  launch_gather<true>(ctx, p, a, SpmvEpi{y}, nullptr);
+  launch_gather<true>(ctx, p, a, SpmvEpi{y}, nullptr, nullptr, nullptr, &p->cb);
 }
 
 void spmv_thread_only(inl_ctx ctx, const inl_csr &A, const float *val, const float *x, float *y) {

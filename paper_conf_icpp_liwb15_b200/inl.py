@@ -24,6 +24,7 @@ INL_OK = 0
 STATUS = {0: "INL_OK", 1: "INL_ERR_INVALID_ARGUMENT", 2: "INL_ERR_OUT_OF_MEMORY", 3: "INL_ERR_CUDA",
           4: "INL_ERR_NCCL", 5: "INL_ERR_NOT_INITIALIZED", 6: "INL_ERR_UNSUPPORTED", 7: "INL_ERR_INTERNAL"}
 BINS_THREAD_ONLY = 1
+BINS_COLBLOCK = 2
 
 
 class InlError(RuntimeError):
@@ -50,7 +51,9 @@ class PlanInfoT(C.Structure):
     _fields_ = [("n_tiles", C.c_int64), ("rows_thread", C.c_int64), ("rows_warp", C.c_int64),
                 ("rows_block", C.c_int64), ("rows_grid", C.c_int64), ("nnz_thread", C.c_int64),
                 ("nnz_warp", C.c_int64), ("nnz_block", C.c_int64), ("nnz_grid", C.c_int64),
-                ("n_grid_chunks", C.c_int64), ("bins", BinsT)]
+                ("n_grid_chunks", C.c_int64), ("bins", BinsT), ("cb_rows", C.c_int64),
+                ("cb_runs", C.c_int64), ("cb_nnz", C.c_int64), ("cb_width", C.c_int64),
+                ("cb_threshold", C.c_int64)]
 
 
 _lib = None

@@ -5,7 +5,7 @@
 //   (2) both at once (half of each lane's gathers on each path).
 // Question it answers: does the TMA unit give SpMV's cold x[col] gathers a second path
 // around the L1TEX wavefront limit?
-// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tma_gather tma_gather.cu
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tma_gather tma_gather.cu -lcuda
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
@@ -23,9 +23,9 @@
   } while (0)
 
 constexpr int W = 16;      // warps per CTA
-constexpr int S = 4;       // pipeline stages per warp
-constexpr int G = 2;       // gather4 per lane per stage
-constexpr int PITCH = 80;  // bytes per lane-group of 4 rows (64 B + 16 B pad: conflict-free LDS)
+constexpr int S = 3;       // pipeline stages per warp
+constexpr int G = 1;       // gather4 per lane per stage (smem: W*S*32*G*PITCH <= 227 KB)
+constexpr int PITCH = 128;  // bytes per lane-group of 4 rows (TMA destinations are 128-B aligned)
 
 __device__ __forceinline__ uint32_t hash32(uint32_t x) {
   x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
@@ -55,7 +55,7 @@ __device__ __forceinline__ void gather4(uint32_t dst, const CUtensorMap *tm, uin
       : "memory");
 }
 
-// MODE 0: LDG only; MODE 1: TMA only; MODE 2: half / half
+// MODE 0: LDG only; MODE 1: TMA only; MODE 2: half / half; MODE 3: TMA, values not read
 template <int MODE>
 __global__ void __launch_bounds__(W * 32, 1) k_bench(const __grid_constant__ CUtensorMap tm, const float *x,
                                                      uint32_t n, int iters, float *out) {
@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(W * 32, 1) k_bench(const __grid_constant__ CUt
 #pragma unroll
         for (int g = 0; g < G; ++g)
 #pragma unroll
-          for (int q = 0; q < 4; ++q) {
+          for (int q = 0; q < (MODE == 3 ? 0 : 4); ++q) {
             float t;
             const uint32_t a = buf + (uint32_t)((s * G + g) * 32 + lane) * PITCH + q * 16 + sel[s][4 * g + q] * 4;
             asm volatile("ld.shared.f32 %0, [%1];" : "=f"(t) : "r"(a));
@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(W * 32, 1) k_bench(const __grid_constant__ CUt
 
 int main(int argc, char **argv) {
   const uint32_t n = argc > 1 ? (uint32_t)atol(argv[1]) : (1u << 22);
-  const int iters = 512;  // stages per warp
+  const int iters = 510;  // stages per warp (a multiple of S)
   int sms = 0, clk = 0;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
   CK(cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, 0));
@@ -149,9 +149,7 @@ int main(int argc, char **argv) {
   CK(cudaMalloc(&x, (size_t)n * 4));
   CK(cudaMemset(x, 0, (size_t)n * 4));
   CK(cudaMalloc(&out, 4));
-  PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
-  cudaDriverEntryPointQueryResult q;
-  CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void **)&enc, cudaEnableDefault, &q));
+  auto enc = cuTensorMapEncodeTiled;
   CUtensorMap tm;
   cuuint64_t dims[2] = {4, n / 4};
   cuuint64_t strides[1] = {16};
@@ -186,5 +184,6 @@ int main(int argc, char **argv) {
   run(k_bench<0>, "ldg", (double)iters * 4 * G);
   run(k_bench<1>, "tma", (double)iters * 4 * G);
   run(k_bench<2>, "ldg+tma", (double)iters * 8 * G);
+  run(k_bench<3>, "tma-noread", (double)iters * 4 * G);
   return 0;
 }
