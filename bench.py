@@ -244,7 +244,7 @@ def run_inl(a):
     reached = []
     # the dominant kernel(s), timed live by the library with events on its own stream
     kernels = (["k_gather", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
-               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up"])
+               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_sssp_split"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
     ctx.ktimer_enable(True)
@@ -295,7 +295,10 @@ def run_inl(a):
         units_local = tot_edges
         relax = sum(r["edges_relaxed"] for r in reached)
         bytes_local = 8 * relax + 16 * sum(r["frontier_total"] for r in reached)
-        launches_per_step = 1 + max(r["iterations"] for r in reached) * 2
+        if all(r.get("launches", 0) > 0 for r in reached):  # counted by the library
+            launches_per_step = sum(r["launches"] for r in reached) / len(reached)
+        else:
+            launches_per_step = 1 + max(r["iterations"] for r in reached) * 2
 
     if a.op in ("spmv", "pagerank"):  # per-step figures -> whole timed region
         units_local *= a.steps
@@ -328,7 +331,7 @@ def run_inl(a):
                        "bins": info["bins"], "plan_ms": round(plan_ms, 3),
                        "l2": "inputs larger than L2 (CSR streamed once per step; L2 is 126 MB)",
                        "thread_only_baseline": bool(a.thread_only)},
-            "gpu_launches": (launches_per_step * a.steps) if launches_per_step else None,
+            "gpu_launches": int(round(launches_per_step * a.steps)) if launches_per_step else None,
         })
         frac = achieved_gbs / peak
         out["roofline"] = {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak, "unit": "GB/s",
@@ -348,6 +351,7 @@ def run_inl(a):
         out["config"]["sources"] = srcs
         out["config"]["iterations"] = [r["iterations"] for r in reached]
         out["config"]["relaxations_per_m_reached"] = round(sum(r["edges_relaxed"] for r in reached) / max(units_total, 1), 3)
+        out["config"]["host_syncs_per_source"] = round(sum(r.get("host_syncs", 0) for r in reached) / max(len(reached), 1), 1)
     if rank == 0:
         out["clocks"] = ck.summary()
         if not a.no_cpu_baseline and world == 1:

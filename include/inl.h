@@ -73,8 +73,9 @@ typedef struct {
  * bench configs) processes SpMV/PR rows of degree > max(t_warp,
  * 4 * column blocks) column-blocked: a CTA holds one block of x in shared memory and
  * sums the row's entries in that block (one partial per (row, block) run, combined in
- * block order). */
-enum { INL_BINS_THREAD_ONLY = 1, INL_BINS_COLBLOCK = 2 };
+ * block order).  INL_BINS_SSSP_DEVLOOP (opt-in, one GPU): the SSSP near-far step loop
+ * runs on the device, the host checks termination every few steps. */
+enum { INL_BINS_THREAD_ONLY = 1, INL_BINS_COLBLOCK = 2, INL_BINS_SSSP_DEVLOOP = 4 };
 typedef struct {
   int32_t t_thread;    /* default 8 */
   int32_t t_warp;      /* default 128, in [16, 4096] (SpMV/PR warp tiles hold < 2*t_warp nnz) */
@@ -88,6 +89,8 @@ typedef struct {
   int32_t iterations;     /* frontier iterations / BFS levels executed */
   int64_t edges_relaxed;  /* sum of the degrees of all frontier vertices expanded */
   int64_t frontier_total; /* sum of frontier sizes over the iterations */
+  int64_t launches;       /* kernels the call launched (memsets and copies excluded) */
+  int64_t host_syncs;     /* host <-> device round trips of the iteration loop */
 } inl_stats;
 
 /* Plan summary (for tests and the bench; counts per bin). */

@@ -18,6 +18,7 @@
 //     BFS allreduce-max of an n-byte next-frontier map, each with a
 //     trailing termination word.
 #include <cooperative_groups.h>
+#include <cstdio>
 #include <cstdlib>
 
 #include <cub/block/block_scan.cuh>
@@ -195,6 +196,31 @@ struct BfsOp {
   }
 };
 
+// Device-driven near-far SSSP (one GPU): the loop state lives on the device, so the
+// host enqueues several steps (split, expand, grid expand, post) per round trip.
+struct __align__(16) SsspDev {
+  int nF;       // input frontier size of this step (0: the step starts with a far split)
+  int cnt;      // next-frontier counter
+  int gcount;   // grid-bin chunk counter
+  int nsplit;   // near vertices the split moved into the frontier
+  int nfar, nfar2;  // far pile sizes (current, split output + this step's far pushes)
+  int par, fpar;    // frontier / far buffer parity
+  int iter, done;
+  uint32_t thr, delta;
+  int slice;    // dynamic slice counter of k_expand_flat
+  int pad;
+  unsigned long long ftotal;
+};
+struct SsspDyn {
+  SsspDev *s;  // nullptr: static (host-driven) launch
+  int32_t *buf[2];
+  int32_t *far[2];
+  uint32_t *inq[2];  // claim bitmaps of even / odd iterations
+  uint32_t *keep;    // in-far-pile bitmap
+};
+
+__device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) { return a > 0xFFFFFFFFu - b ? 0xFFFFFFFFu : a + b; }
+
 struct ExpandArgs {
   const int32_t *F;  // frontier (local row ids)
   int nF;
@@ -206,7 +232,49 @@ struct ExpandArgs {
   int32_t *Fout;
   int *fcount;
   unsigned long long *relaxed;
+  SsspDyn dyn;
 };
+
+// The step state, read once per CTA (4 lanes, 16-B L2 loads) into shared memory: every
+// thread reading it from global memory would hammer one L2 slice.
+__device__ __forceinline__ void load_state(const SsspDev *g, SsspDev *sh) {
+  if (threadIdx.x < (int)(sizeof(SsspDev) / 16))
+    reinterpret_cast<int4 *>(sh)[threadIdx.x] = __ldcg(reinterpret_cast<const int4 *>(g) + threadIdx.x);
+  __syncthreads();
+}
+
+// Dynamic launches read this step's frontier / far-pile / claim-bitmap roles from the
+// device state; returns false when the step has nothing to expand.
+template <class Op>
+__device__ __forceinline__ bool dyn_bind(ExpandArgs &a, Op &op, uint32_t **inq_prev) {
+  *inq_prev = nullptr;
+  return true;
+}
+template <>
+__device__ __forceinline__ bool dyn_bind<SsspOp>(ExpandArgs &a, SsspOp &op, uint32_t **inq_prev) {
+  *inq_prev = nullptr;
+  if (!a.dyn.s) return true;
+  __shared__ __align__(16) SsspDev st_s;
+  load_state(a.dyn.s, &st_s);
+  const SsspDev &s = st_s;
+  if (s.done) return false;
+  const bool split = s.nF == 0;
+  const int nF = split ? s.nsplit : s.nF;
+  if (nF == 0) return false;
+  const int par = s.par, fpar = s.fpar, it = s.iter;
+  a.nF = nF;
+  a.F = a.dyn.buf[par];
+  a.Fout = a.dyn.buf[par ^ 1];
+  a.fcount = &a.dyn.s->cnt;
+  a.gcount = &a.dyn.s->gcount;
+  op.thr = split ? sat_add(s.thr, s.delta) : s.thr;
+  op.inq = a.dyn.inq[it & 1];
+  op.far = a.dyn.far[split ? fpar ^ 1 : fpar];
+  op.far_count = split ? &a.dyn.s->nfar2 : &a.dyn.s->nfar;
+  op.infar = a.dyn.keep;
+  *inq_prev = a.dyn.inq[(it & 1) ^ 1];
+  return true;
+}
 
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
@@ -275,6 +343,8 @@ constexpr int kEdgesPerThread = 8;
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
+  uint32_t *inq_prev;
+  if (!dyn_bind(a, op, &inq_prev)) return;
   using Scan = cub::BlockScan<int, NT>;
   __shared__ typename Scan::TempStorage scan_tmp;
   __shared__ int64_t rs_s[NT];
@@ -282,16 +352,27 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
   __shared__ uint32_t su_s[NT];
   __shared__ unsigned long long red[NW];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int i = blockIdx.x * NT + tid;
+  unsigned long long mydeg = 0;
+  // static launches have one slice of NT frontier vertices per CTA; dynamic ones a fixed
+  // grid whose CTAs take slices from a counter (load balance across the grid)
+  __shared__ int slice_s;
+  int base = blockIdx.x * NT;
+  if (a.dyn.s) {
+    if (tid == 0) slice_s = atomicAdd(&a.dyn.s->slice, 1);
+    __syncthreads();
+    base = slice_s * NT;
+  }
+  while (base < a.nF) {
+  const int i = base + tid;
   int d = 0;
   int64_t rs = 0;
   uint32_t su = 0;
-  unsigned long long mydeg = 0;
   if (i < a.nF) {
     const int32_t u = a.F[i];
+    if (inq_prev) inq_prev[u >> 5] = 0u;  // its claim bit of the previous iteration
     rs = a.rp[u];
     const int64_t dd = a.rp[u + 1] - rs;
-    mydeg = (unsigned long long)dd;
+    mydeg += (unsigned long long)dd;
     su = op.load(u);
     if (dd > a.t_warp) {  // grid bin: global delayed buffer
       const int nch = (int)((dd + a.chunk - 1) / a.chunk);
@@ -349,6 +430,15 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
     for (int j = 0; j < kEdgesPerThread; ++j) vv[j] = in[j] ? (int32_t)ld_stream_pol(a.col + kk[j], op.pol_stream) : 0;
     op.edges(du, kk, vv, in, a.Fout, a.fcount);
   }
+  __syncthreads();  // the run buffer is rewritten by the next slice
+  if (a.dyn.s) {
+    if (tid == 0) slice_s = atomicAdd(&a.dyn.s->slice, 1);
+    __syncthreads();
+    base = slice_s * NT;
+  } else {
+    base += gridDim.x * NT;
+  }
+  }
   for (int o = 16; o > 0; o >>= 1) mydeg += __shfl_xor_sync(0xffffffffu, mydeg, o);
   if (lane == 0) red[warp] = mydeg;
   __syncthreads();
@@ -364,7 +454,12 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
-  const int n = *(volatile int *)a.gcount;
+  uint32_t *inq_prev;
+  if (!dyn_bind(a, op, &inq_prev)) return;
+  __shared__ int n_s;  // one L2 read per CTA (every thread reading it would hit one L2 slice)
+  if (threadIdx.x == 0) n_s = __ldcg(a.gcount);
+  __syncthreads();
+  const int n = n_s;
   for (int it = blockIdx.x; it < n; it += gridDim.x) {
     const int2 g = a.gitems[it];
     const int64_t rs = a.rp[g.x], re = a.rp[g.x + 1];
@@ -420,6 +515,58 @@ __global__ void k_far_split(const int32_t *__restrict__ far, int nfar, const uin
       if (!(atomicOr(keep + (v >> 5), bit) & bit)) push(far2, far2cnt, v);
     }
   }
+}
+
+// Device-driven step, part 1: when the near frontier is empty, advance the threshold and
+// split the far pile (duplicate-free): lo <= dist < hi -> frontier, dist >= hi -> the other
+// far buffer (stays marked in `keep`), dist < lo -> settled earlier, dropped.
+__global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) {
+  __shared__ __align__(16) SsspDev st_s;
+  load_state(dy.s, &st_s);
+  const SsspDev *s = &st_s;
+  if (s->done || s->nF != 0) return;
+  const int nfar = s->nfar;
+  if (nfar == 0) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) dy.s->done = 1;
+    return;
+  }
+  const uint32_t lo = s->thr, hi = sat_add(lo, s->delta);
+  const int fpar = s->fpar, par = s->par;
+  const int32_t *far = dy.far[fpar];
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nfar; i += gridDim.x * blockDim.x) {
+    const int32_t v = far[i];
+    const uint32_t d = dist[v];
+    if (d >= hi) {
+      push(dy.far[fpar ^ 1], &dy.s->nfar2, v);
+    } else {
+      atomicAnd(dy.keep + (v >> 5), ~(1u << (v & 31)));
+      if (d >= lo) push(dy.buf[par], &dy.s->nsplit, v);
+    }
+  }
+}
+
+// Device-driven step, part 4: roll the state over to the next step.
+__global__ void k_sssp_post(SsspDyn dy) {
+  SsspDev *s = dy.s;
+  if (s->done) return;
+  const bool split = s->nF == 0;
+  if (split) {
+    s->thr = sat_add(s->thr, s->delta);
+    s->nfar = s->nfar2;
+    s->nfar2 = 0;
+    s->fpar ^= 1;
+  }
+  const int size = split ? s->nsplit : s->nF;
+  s->nsplit = 0;
+  if (size > 0) {
+    s->ftotal += (unsigned long long)size;
+    s->iter += 1;
+    s->nF = s->cnt;
+    s->par ^= 1;
+  }
+  s->cnt = 0;
+  s->gcount = 0;
+  s->slice = 0;
 }
 
 // P > 1: vertices of the owned slice whose distance dropped -> next frontier.
@@ -587,15 +734,106 @@ void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_
   st->iterations = iters;
   st->edges_relaxed = (int64_t)r;
   st->frontier_total = ftotal;
+  st->launches = 0;  // host-driven loops: not counted
+  st->host_syncs = iters;
 }
 
 }  // namespace
+
+// One GPU, near-far: the step loop runs on the device (k_sssp_split, k_expand_flat,
+// k_expand_grid, k_sssp_post per step, fixed grids); the host enqueues `batch` steps per
+// round trip and reads back the `done` flag.  Same fixed point as the host-driven loop.
+static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
+                         uint32_t *dist, inl_stats *stats) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = G.n_global;
+  FrontierBufs f = frontier_bufs(ctx, G, b);
+  INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
+  const int64_t nwb = (n + 31) / 32 + 1;
+  SsspDyn dy;
+  uint32_t *bits = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 3 * nwb);
+  dy.inq[0] = bits;
+  dy.inq[1] = bits + nwb;
+  dy.keep = bits + 2 * nwb;
+  INL_CUDA(cudaMemsetAsync(bits, 0, sizeof(uint32_t) * 3 * nwb, st));
+  dy.far[0] = (int32_t *)ctx->s_g.get(sizeof(int32_t) * (2 * n + 16));
+  dy.far[1] = dy.far[0] + n + 8;
+  dy.buf[0] = f.F;
+  dy.buf[1] = f.Fout;
+  dy.s = (SsspDev *)ctx->s_e.get(sizeof(SsspDev));
+  static_assert(sizeof(SsspDev) <= 64, "SsspDev is read back through the ctx's 64-B pinned buffer");
+  const bool owned = source >= G.row_begin && source < G.row_begin + G.n_rows;
+  SsspDev h{};
+  h.nF = owned ? 1 : 0;
+  h.thr = h.delta = sssp_delta();
+  INL_CUDA(cudaMemcpyAsync(dy.s, &h, sizeof h, cudaMemcpyHostToDevice, st));
+  const int32_t s0 = (int32_t)(owned ? source - G.row_begin : 0);
+  INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(dist, n, source);
+  INL_CUDA(cudaGetLastError());
+  ExpandArgs a{f.F, 0, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
+               f.gitems, nullptr, f.Fout, nullptr, f.relaxed};
+  a.dyn = dy;
+  SsspOp op{dist, w, nullptr, nullptr, 0, 0, true, 0, 0, nullptr, nullptr, nullptr};
+  static int gmul = -1;  // grid multipliers (env INL_SSSP_GRIDS=split,flat,grid for tuning)
+  static int gm[3] = {2, 8, 2};
+  if (gmul < 0) {
+    gmul = 1;
+    if (const char *e = getenv("INL_SSSP_GRIDS")) sscanf(e, "%d,%d,%d", &gm[0], &gm[1], &gm[2]);
+  }
+  const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
+  int64_t launches = 1, syncs = 0;
+  int batch = 4;
+  SsspDev *hs = (SsspDev *)ctx->pinned;  // pinned scratch (>= 64 B)
+  for (;;) {
+    for (int k = 0; k < batch; ++k) {
+      {
+        KScope ks(ctx, "k_sssp_split");
+        k_sssp_split<<<gsplit, 256, 0, st>>>(dy, dist);
+      }
+      {
+        KScope ks(ctx, "k_expand_flat");
+        k_expand_flat<SsspOp><<<gflat, NT, 0, st>>>(a, op);
+      }
+      {
+        KScope ks(ctx, "k_expand_grid");
+        k_expand_grid<SsspOp><<<ggrid, NT, 0, st>>>(a, op);
+      }
+      k_sssp_post<<<1, 1, 0, st>>>(dy);
+      launches += 4;
+    }
+    INL_CUDA(cudaGetLastError());
+    INL_CUDA(cudaMemcpyAsync(hs, dy.s, sizeof(SsspDev), cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    ++syncs;
+    if (((volatile SsspDev *)hs)->done) break;
+    if (batch < 16) batch *= 2;
+  }
+  if (stats) {
+    unsigned long long r = 0;
+    INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    stats->iterations = hs->iter;
+    stats->edges_relaxed = (int64_t)r;
+    stats->frontier_total = (int64_t)hs->ftotal;
+    stats->launches = launches;
+    stats->host_syncs = syncs;
+  }
+}
 
 void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
               uint32_t *dist, inl_stats *stats) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  // the device-driven loop (sssp_run_dyn) is opt-in: measured 8.5 ms vs 8.0 ms per scale-23
+  // source for the host-driven one (profiles/r01/sssp_devloop.txt) — its 4 launches per
+  // step cost more than the ~40 host round trips they save
+  const bool devloop = (b.flags & INL_BINS_SSSP_DEVLOOP) != 0;
+  if (!DIST && !(b.flags & INL_BINS_THREAD_ONLY) && devloop && sssp_delta() != 0xFFFFFFFFu && n > 0) {
+    sssp_run_dyn(ctx, G, b, w, source, dist, stats);
+    return;
+  }
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
   uint32_t *D = dist;

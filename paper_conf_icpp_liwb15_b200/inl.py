@@ -25,6 +25,7 @@ STATUS = {0: "INL_OK", 1: "INL_ERR_INVALID_ARGUMENT", 2: "INL_ERR_OUT_OF_MEMORY"
           4: "INL_ERR_NCCL", 5: "INL_ERR_NOT_INITIALIZED", 6: "INL_ERR_UNSUPPORTED", 7: "INL_ERR_INTERNAL"}
 BINS_THREAD_ONLY = 1
 BINS_COLBLOCK = 2
+BINS_SSSP_DEVLOOP = 4
 
 
 class InlError(RuntimeError):
@@ -44,7 +45,8 @@ class BinsT(C.Structure):
 
 
 class StatsT(C.Structure):
-    _fields_ = [("iterations", C.c_int32), ("edges_relaxed", C.c_int64), ("frontier_total", C.c_int64)]
+    _fields_ = [("iterations", C.c_int32), ("edges_relaxed", C.c_int64), ("frontier_total", C.c_int64),
+                ("launches", C.c_int64), ("host_syncs", C.c_int64)]
 
 
 class PlanInfoT(C.Structure):
@@ -296,7 +298,8 @@ def sssp(ctx: Ctx, G: Csr, w, source: int, dist, plan: Plan | None = None) -> di
     st = StatsT()
     _check(lib().inl_sssp(ctx.handle, C.byref(s), _ptr(w), int(source), _ptr(dist), C.byref(st),
                           _plan_handle(plan)), ctx)
-    return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total}
+    return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total,
+            "launches": st.launches, "host_syncs": st.host_syncs}
 
 
 def bfs(ctx: Ctx, G: Csr, source: int, level, plan: Plan | None = None) -> dict:
@@ -306,4 +309,5 @@ def bfs(ctx: Ctx, G: Csr, source: int, level, plan: Plan | None = None) -> dict:
     st = StatsT()
     _check(lib().inl_bfs(ctx.handle, C.byref(s), int(source), _ptr(level), C.byref(st),
                          _plan_handle(plan)), ctx)
-    return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total}
+    return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total,
+            "launches": st.launches, "host_syncs": st.host_syncs}

@@ -48,7 +48,9 @@ def gpu_bfs(ctx, rp, ci, n, s, b=None):
 
 BINS = [None, dict(t_thread=-1, t_warp=32, t_block=128, grid_chunk=64),
         dict(t_thread=1, t_warp=128, t_block=256, grid_chunk=64), dict(flags=inl.BINS_THREAD_ONLY),
-        dict(t_thread=64, t_warp=128, t_block=4096, grid_chunk=1000)]
+        dict(t_thread=64, t_warp=128, t_block=4096, grid_chunk=1000),
+        dict(flags=inl.BINS_SSSP_DEVLOOP),  # device-driven near-far step loop
+        dict(t_thread=1, t_warp=32, t_block=128, grid_chunk=64, flags=inl.BINS_SSSP_DEVLOOP)]
 
 
 @pytest.mark.parametrize("bi", range(len(BINS)))
@@ -81,6 +83,27 @@ def test_small_graph_edge_cases(ctx):
         assert np.array_equal(d, oracle.sssp(rp, ci, w, s))
         lv, _ = gpu_bfs(ctx, rp, ci, n, s)
         assert np.array_equal(lv, oracle.bfs(rp, ci, s))
+
+
+def test_devloop_edge_cases_and_certificate(ctx):
+    b = inl.bins(flags=inl.BINS_SSSP_DEVLOOP)
+    rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3), (3, 1)], [5, 6, 7], symmetric=True)
+    d, st = gpu_sssp(ctx, rp, ci, w, 6, 0, b)  # isolated source
+    assert d.tolist() == [0] + [0xFFFFFFFF] * 5 and st["host_syncs"] >= 1
+    n = 30000
+    e = [(0, i) for i in range(1, n - 100)] + [(i, i + 1) for i in range(n - 101, n - 1)]
+    rp, ci, w = csr_from_edges(n, e, np.arange(len(e)) % 255 + 1, symmetric=True)
+    for s in (0, n - 1, 5):
+        d, _ = gpu_sssp(ctx, rp, ci, w, n, s, b)
+        assert np.array_equal(d, oracle.sssp(rp, ci, w, s))
+    g = inlgen.host_build(16, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    w = inlgen.weights_host(g.row_ptr, g.col_idx)
+    for s in inlgen.sources(g.row_ptr, 3):
+        d, st = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, b)
+        assert certify_sssp(g.row_ptr, g.col_idx, w, s, d) is None
+        ref, st0 = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, inl.bins())
+        assert np.array_equal(d, ref)
+        assert st["launches"] > 0 and st["host_syncs"] < st0["host_syncs"]
 
 
 def test_host_buffers(ctx, cfg1):
