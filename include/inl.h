@@ -75,13 +75,24 @@ typedef struct {
  * sums the row's entries in that block (one partial per (row, block) run, combined in
  * block order).  INL_BINS_SSSP_DEVLOOP (opt-in, one GPU): the SSSP near-far step loop
  * runs on the device, the host checks termination every few steps. */
-enum { INL_BINS_THREAD_ONLY = 1, INL_BINS_COLBLOCK = 2, INL_BINS_SSSP_DEVLOOP = 4 };
+enum {
+  INL_BINS_THREAD_ONLY = 1,
+  INL_BINS_COLBLOCK = 2,
+  INL_BINS_SSSP_DEVLOOP = 4,
+  /* The paper's templates, as it describes them (SpMV only; template study):
+   * lbTHRES = t_thread (rows of degree > t_thread are block-mapped), CTA = cta_threads.
+   * dual-queue (Fig. 1(b), P5@2074), dbuf-global and dbuf-shared (Fig. 1(c), P5@2717). */
+  INL_BINS_TPL_DUAL_QUEUE = 8,
+  INL_BINS_TPL_DBUF_GLOBAL = 16,
+  INL_BINS_TPL_DBUF_SHARED = 32
+};
 typedef struct {
   int32_t t_thread;    /* default 8 */
   int32_t t_warp;      /* default 128, in [16, 4096] (SpMV/PR warp tiles hold < 2*t_warp nnz) */
   int32_t t_block;     /* default 16384, >= t_warp */
-  int32_t grid_chunk;  /* default 4096 nnz per block/grid-bin piece (one warp each), in [32, 2^20] */
-  int32_t cta_threads; /* reserved (128/256/512 accepted); kernels use fixed CTA shapes */
+  int32_t grid_chunk;  /* default 8192 nnz per block/grid-bin piece (one warp each), in [32, 2^20] */
+  int32_t cta_threads; /* CTA size of the INL_BINS_TPL_* templates (multiple of 32 in [32, 1024],
+                          default 256); the default kernels use fixed CTA shapes */
   int32_t flags;
 } inl_bins;
 

@@ -88,7 +88,7 @@ KTimer::~KTimer() {
 }
 
 Bins resolve_bins(const inl_bins *b) {
-  Bins r{8, 1024, 16384, 4096, 256, 0};
+  Bins r{8, 1024, 16384, 8192, 256, 0};
   if (b) {
     if (b->t_thread > 0) r.t_thread = b->t_thread;
     if (b->t_thread < 0) r.t_thread = 0;
@@ -98,7 +98,7 @@ Bins resolve_bins(const inl_bins *b) {
     if (b->cta_threads > 0) r.cta = b->cta_threads;
     r.flags = b->flags;
   }
-  INL_CHECK(r.cta == 128 || r.cta == 256 || r.cta == 512, "bins.cta_threads must be 128, 256 or 512");
+  INL_CHECK(r.cta >= 32 && r.cta <= 1024 && r.cta % 32 == 0, "bins.cta_threads must be a multiple of 32 in [32, 1024]");
   INL_CHECK(r.t_thread <= r.t_warp && r.t_warp <= r.t_block,
             "bins: need t_thread <= t_warp <= t_block");
   INL_CHECK(r.t_warp >= 16 && r.t_warp <= 4096, "bins.t_warp must be in [16, 4096]");
@@ -448,7 +448,8 @@ inl_status inl_plan_create(inl_ctx ctx, const inl_csr *A, const inl_bins *bins, 
     p->row_ptr = A->row_ptr;
     p->col_idx = A->col_idx;
     p->bins = resolve_bins(bins);
-    if (!(p->bins.flags & INL_BINS_THREAD_ONLY)) build_plan(p);  // the T1 baseline needs no bins
+    if (!(p->bins.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)))
+      build_plan(p);  // the T1 baseline and the paper's templates need no bins
   });
   if (s != INL_OK) {
     delete p;
@@ -504,6 +505,9 @@ inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float
     if (plan && (plan->bins.flags & INL_BINS_THREAD_ONLY)) {
       INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
       spmv_thread_only(ctx, d, dval, dx, yo.dev);
+    } else if (plan && (plan->bins.flags & kTemplateFlags)) {
+      INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
+      spmv_template(ctx, d, plan->bins, dval, dx, yo.dev);
     } else {
       PlanHolder tmp;
       inl_plan p = get_plan(ctx, d, plan, &tmp.p);
@@ -533,6 +537,8 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
     StagedOut<float> ro = stage_out(ctx->h_y, rank, A_in->n_global);
     if (plan && (plan->bins.flags & INL_BINS_THREAD_ONLY))
       raise(INL_ERR_UNSUPPORTED, "thread-only baseline plans are SpMV/SSSP/BFS only");
+    if (plan && (plan->bins.flags & kTemplateFlags))
+      raise(INL_ERR_UNSUPPORTED, "paper-template plans (INL_BINS_TPL_*) are SpMV only");
     PlanHolder tmp;
     inl_plan p = get_plan(ctx, d, plan, &tmp.p);
     pagerank_run(ctx, p, dod, damping, iterations, ro.dev);

@@ -443,7 +443,7 @@ __global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, Gath
 
 // x_hot[h] = x[hot_cols[h]] (per call; zero-padded to a multiple of 4) — spmv.cu.
 // hot_cols: NULL = the plan's list, else a list in another column space.
-void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols = nullptr);
+void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols = nullptr, int64_t n_hot = -1);
 
 template <int E, bool VALS, class Epi, int NWARP = 256 / E>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
@@ -479,8 +479,9 @@ inline int gather_entries_per_lane() {
 template <bool VALS, class Epi>
 void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart,
                    const int32_t *col_over = nullptr, const int32_t *hot_over = nullptr,
-                   const CbPlan *cb = nullptr) {
+                   const CbPlan *cb = nullptr, int64_t n_hot_over = -1) {
   if (p->n_items == 0) return;
+  const int64_t n_hot = n_hot_over >= 0 ? n_hot_over : p->n_hot;
   const bool use_cb = cb && cb->active;
   const int64_t n_items = use_cb ? cb->n_items : p->n_items;
   GatherArgs a = a_in;
@@ -494,7 +495,7 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     gp.tickets = (int *)p->tickets.p;
     gp.dpart = dpart;
     gp.x_hot = (const float *)p->x_hot.p;
-    gp.n_hot = (int)((p->n_hot + 3) & ~3);
+    gp.n_hot = (int)((n_hot + 3) & ~3);
     gp.rs_bits = (const uint32_t *)p->rs_bits.p;
     gp.tile_nz = (const uint32_t *)p->tile_nz.p;
     gp.ticket = (unsigned long long *)p->ticket.p;
@@ -502,7 +503,7 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     // grab per active warp), so the next launch's base is known on the host: no reset
     gp.base = p->ticket_base;
     p->ticket_base += (unsigned long long)n_items;
-    build_xhot(ctx, p, a.x, hot_over);
+    build_xhot(ctx, p, a.x, hot_over, n_hot);
     a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
     static int w24 = -1;
     if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;

@@ -180,7 +180,8 @@ struct inl_plan_s {
   int64_t pr_bc = 0;           // compact slots per rank block
   inl::DevBuf pr_cidx;         // int32 [n_global]: exchange-space index, -1 if dangling
   inl::DevBuf pr_col;          // int32 [nnz]: gather columns in the compact space (hot kept)
-  inl::DevBuf pr_hot;          // int32 [n_hot]: hot slots in the compact space
+  inl::DevBuf pr_hot;          // int32 [pr_nhot]: hot slots in the compact space
+  int64_t pr_nhot = 0;         // PageRank's hot slots (a prefix of the plan's)
   // column-blocked long rows: SpMV (the CSR's column space) and PageRank (compact space)
   inl::CbPlan cb, pr_cb;
 };
@@ -217,6 +218,9 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
               uint32_t *dist, inl_stats *st);
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
              inl_stats *st);
+// templates.cu: the paper's dual-queue / dbuf-global / dbuf-shared SpMV (false: no template flag)
+constexpr int kTemplateFlags = INL_BINS_TPL_DUAL_QUEUE | INL_BINS_TPL_DBUF_GLOBAL | INL_BINS_TPL_DBUF_SHARED;
+bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *val, const float *x, float *y);
 // colblock.cu: builds `cb` for the column space `cols` (raw ids in [0, ncols), CSR order)
 void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool sort_rows = false);
 // validate

@@ -112,10 +112,12 @@ __global__ void k_cidx_sorted(const int32_t *__restrict__ od, const int32_t *__r
 // gather columns in the compact space (hot slots kept); a column without out-links
 // (inconsistent input) reads the zero slot
 __global__ void k_remap_cols(const int32_t *__restrict__ col, int64_t nnz, const int32_t *__restrict__ cidx,
-                             int32_t zero_slot, int32_t *__restrict__ out) {
+                             int32_t zero_slot, int32_t *__restrict__ out, const int32_t *__restrict__ hot_cols = nullptr,
+                             int n_hot = 0) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz;
        k += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t c = col[k];
+    int32_t c = col[k];
+    if (c < 0 && (c & 0x7FFFFFFF) >= n_hot) c = hot_cols[c & 0x7FFFFFFF];  // beyond PageRank's hot set
     if (c < 0) {
       out[k] = c;
     } else {
@@ -190,11 +192,21 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
   const int32_t zero_slot = (int32_t)(bc * P);
   const int32_t *src = p->n_hot > 0 ? (const int32_t *)p->pcol.p : p->col_idx;
   int32_t *pc = (int32_t *)p->pr_col.get(sizeof(int32_t) * (p->nnz > 0 ? p->nnz : 1));
+  // PageRank's own hot set: the first pr_nhot slots of the plan's (ranked by frequency);
+  // fewer than SpMV's because the contribution gathers miss L2 more often and profit from
+  // the L1 capacity a smaller shared-memory copy leaves (measured, profiles/r01)
+  int64_t nh = 16384;
+  if (const char *e = getenv("INL_PR_HOT_K")) nh = atoll(e);
+  if (nh > p->n_hot) nh = p->n_hot;
+  if (nh < 0) nh = 0;
+  p->pr_nhot = nh & ~(int64_t)3;
+  if (p->n_hot > 0 && p->pr_nhot < 4) p->pr_nhot = 0;
   if (p->nnz > 0)
-    k_remap_cols<<<grid_for(p->nnz, ctx->num_sms), 256, 0, st>>>(src, p->nnz, cidx, zero_slot, pc);
-  if (p->n_hot > 0) {
-    int32_t *ph = (int32_t *)p->pr_hot.get(sizeof(int32_t) * p->n_hot);
-    k_remap_hot<<<grid_for(p->n_hot, ctx->num_sms), 256, 0, st>>>((const int32_t *)p->hot_cols.p, (int)p->n_hot,
+    k_remap_cols<<<grid_for(p->nnz, ctx->num_sms), 256, 0, st>>>(src, p->nnz, cidx, zero_slot, pc,
+                                                                 (const int32_t *)p->hot_cols.p, (int)p->pr_nhot);
+  if (p->pr_nhot > 0) {
+    int32_t *ph = (int32_t *)p->pr_hot.get(sizeof(int32_t) * p->pr_nhot);
+    k_remap_hot<<<grid_for(p->pr_nhot, ctx->num_sms), 256, 0, st>>>((const int32_t *)p->hot_cols.p, (int)p->pr_nhot,
                                                                  cidx, zero_slot, ph);
   }
   INL_CUDA(cudaGetLastError());
@@ -253,7 +265,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
     PrEpi epi{out_degree, c_next, cidx, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
               p->row_begin, 0.0f};
     launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p,
-                         p->n_hot > 0 ? (const int32_t *)p->pr_hot.p : nullptr, &p->pr_cb);
+                         p->pr_nhot > 0 ? (const int32_t *)p->pr_hot.p : nullptr, &p->pr_cb, p->pr_nhot);
     if (!last) {
       k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
       INL_CUDA(cudaGetLastError());

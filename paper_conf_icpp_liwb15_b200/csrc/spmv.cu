@@ -11,9 +11,9 @@ __global__ void k_build_xhot(const float *__restrict__ x, const int32_t *__restr
 }
 }  // namespace
 
-void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols) {
-  if (p->n_hot == 0) return;
-  const int n = (int)p->n_hot;
+void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols, int64_t n_hot) {
+  const int n = (int)(n_hot >= 0 ? n_hot : p->n_hot);
+  if (n == 0) return;
   k_build_xhot<<<(n + 255) / 256, 256, 0, ctx->stream>>>(
       x, hot_cols ? hot_cols : (const int32_t *)p->hot_cols.p, n, (float *)p->x_hot.p);
   INL_CUDA(cudaGetLastError());

@@ -26,6 +26,9 @@ STATUS = {0: "INL_OK", 1: "INL_ERR_INVALID_ARGUMENT", 2: "INL_ERR_OUT_OF_MEMORY"
 BINS_THREAD_ONLY = 1
 BINS_COLBLOCK = 2
 BINS_SSSP_DEVLOOP = 4
+BINS_TPL_DUAL_QUEUE = 8
+BINS_TPL_DBUF_GLOBAL = 16
+BINS_TPL_DBUF_SHARED = 32
 
 
 class InlError(RuntimeError):

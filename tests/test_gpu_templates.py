@@ -1,0 +1,81 @@
+"""GPU parity of the paper's load-balancing templates (templates.cu) vs the oracle.
+
+dual-queue (Fig. 1(b), P5@2074), dbuf-global and dbuf-shared (Fig. 1(c), P5@2717,
+P5@3623) for SpMV, over lbTHRES (P5@332) and CTA sizes (P5@11808, P11@1656).
+Bar: integer-valued SpMV bit-exact; fp32 max relative error <= 1e-5.
+"""
+import numpy as np
+import pytest
+import torch
+
+import inlgen
+import oracle
+from graphs import csr_from_edges
+from paper_conf_icpp_liwb15_b200 import inl
+
+pytestmark = pytest.mark.gpu
+TPL = {"dual_queue": inl.BINS_TPL_DUAL_QUEUE, "dbuf_global": inl.BINS_TPL_DBUF_GLOBAL,
+       "dbuf_shared": inl.BINS_TPL_DBUF_SHARED}
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    return inl.Ctx(0)
+
+
+@pytest.fixture(scope="module")
+def g14():
+    return inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH)
+
+
+def run(ctx, rp, ci, n, val, x, flags, lbt, cta):
+    A = inl.Csr(dev(rp), dev(ci), n)
+    plan = inl.Plan(ctx, A, inl.bins(t_thread=lbt if lbt > 0 else -1, t_warp=max(lbt, 16),
+                                      t_block=max(lbt, 16), cta_threads=cta, flags=flags))
+    y = torch.full((len(rp) - 1,), float("nan"), device="cuda")
+    inl.spmv(ctx, A, dev(val), dev(x), y, plan)
+    torch.cuda.synchronize()
+    return y.cpu().numpy().astype(np.float64)
+
+
+@pytest.mark.parametrize("name", sorted(TPL))
+@pytest.mark.parametrize("lbt,cta", [(0, 64), (8, 192), (32, 256), (128, 64), (1024, 1024)])
+def test_template_integer_bit_exact(ctx, g14, name, lbt, cta):
+    val = inlgen.values_host(g14.row_ptr, g14.col_idx, mode=1)
+    x = inlgen.vector_host(g14.n_global, mode=1)
+    ref = oracle.spmv(g14.row_ptr, g14.col_idx, val, x)
+    y = run(ctx, g14.row_ptr, g14.col_idx, g14.n_global, val, x, TPL[name], lbt, cta)
+    assert np.array_equal(y, ref)
+
+
+@pytest.mark.parametrize("name", sorted(TPL))
+def test_template_uniform_and_star(ctx, g14, name):
+    val = inlgen.values_host(g14.row_ptr, g14.col_idx)
+    x = inlgen.vector_host(g14.n_global)
+    ref = oracle.spmv(g14.row_ptr, g14.col_idx, val, x)
+    y = run(ctx, g14.row_ptr, g14.col_idx, g14.n_global, val, x, TPL[name], 32, 192)
+    nz = ref != 0
+    assert np.all(y[~nz] == 0) and np.max(np.abs(y[nz] - ref[nz]) / ref[nz]) <= 1e-5
+    # one row far above lbTHRES among empty and short rows
+    n = 5000
+    e = [(0, i) for i in range(1, n)] + [(i, (i * 7) % n) for i in range(2, n, 3)]
+    rp, ci, w = csr_from_edges(n, e, np.ones(len(e), np.uint32), symmetric=False)
+    v = (np.arange(len(ci)) % 5 + 1).astype(np.float32)
+    xx = (np.arange(n) % 3).astype(np.float32)
+    assert np.array_equal(run(ctx, rp, ci, n, v, xx, TPL[name], 16, 64), oracle.spmv(rp, ci, v, xx))
+
+
+def test_template_flags_are_spmv_only(ctx, g14):
+    A = inl.Csr(dev(g14.row_ptr), dev(g14.col_idx), g14.n_global)
+    plan = inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DBUF_SHARED))
+    r = torch.empty(g14.n_global, device="cuda")
+    with pytest.raises(RuntimeError):
+        inl.pagerank(ctx, A, dev(np.ones(g14.n_global, np.int32)), r, 0.85, 2, plan)
+    both = inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DUAL_QUEUE))
+    y = torch.empty(g14.n_rows, device="cuda")
+    with pytest.raises(RuntimeError):
+        inl.spmv(ctx, A, dev(np.ones(g14.nnz, np.float32)), dev(np.ones(g14.n_global, np.float32)), y, both)
