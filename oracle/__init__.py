@@ -29,6 +29,7 @@ def lib() -> C.CDLL:
         L.orc_pagerank.argtypes = [i64, vp, vp, vp, C.c_double, C.c_int32, vp]
         L.orc_sssp_dijkstra.argtypes = [i64, vp, vp, vp, i64, vp]
         L.orc_bfs.argtypes = [i64, vp, vp, i64, vp]
+        L.orc_bc.argtypes = [i64, vp, vp, vp, i64, vp]
         _lib = L
     return _lib
 
@@ -80,3 +81,15 @@ def bfs(row_ptr, col_idx, source) -> np.ndarray:
     lv = np.empty(n, dtype=np.int32)
     _rc(lib().orc_bfs(n, prp, pci, source, lv.ctypes.data), "orc_bfs")
     return lv
+
+
+def bc(row_ptr, col_idx, sources=None) -> np.ndarray:
+    """Betweenness over the given sources (None = all vertices: exact BC), fp64."""
+    rp, prp = _a(row_ptr, np.int64)
+    ci, pci = _a(col_idx, np.int32)
+    n = len(rp) - 1
+    src = np.arange(n, dtype=np.int64) if sources is None else np.ascontiguousarray(sources, dtype=np.int64)
+    out = np.empty(n, dtype=np.float64)
+    _rc(lib().orc_bc(n, prp, pci, src.ctypes.data if src.size else 0, len(src), out.ctypes.data if n else 0),
+        "orc_bc")
+    return out

@@ -173,3 +173,63 @@ int orc_bfs(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t s
   free(queue);
   return 0;
 }
+
+/* Betweenness centrality: Brandes, "A faster algorithm for betweenness centrality"
+ * (J. Math. Sociol. 2001), Algorithm 1 for unweighted graphs, the method the paper's [6]
+ * parallelises (P5@8911: "First, it constructs the shortest paths tree using BFS ...;
+ * second, it computes the BC value by traversing the shortest path tree").  Per source:
+ * FIFO BFS recording sigma (shortest-path counts) and the visit order S; then vertices in
+ * reverse visit order accumulate delta; bc[w] += delta[w] for w != s. */
+int orc_bc(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int64_t *sources,
+           int64_t n_sources, double *bc) {
+  if (n < 0 || n_sources < 0 || !row_ptr || (n > 0 && !bc) || (n_sources > 0 && !sources)) return -1;
+  for (int64_t i = 0; i < n_sources; ++i)
+    if (sources[i] < 0 || sources[i] >= n) return -1;
+  for (int64_t v = 0; v < n; ++v) bc[v] = 0.0;
+  if (n == 0) return 0;
+  int64_t *S = (int64_t *)malloc(sizeof(int64_t) * (size_t)n);
+  int64_t *dist = (int64_t *)malloc(sizeof(int64_t) * (size_t)n);
+  double *sigma = (double *)malloc(sizeof(double) * (size_t)n);
+  double *delta = (double *)malloc(sizeof(double) * (size_t)n);
+  if (!S || !dist || !sigma || !delta) {
+    free(S); free(dist); free(sigma); free(delta);
+    return -2;
+  }
+  for (int64_t i = 0; i < n_sources; ++i) {
+    const int64_t s = sources[i];
+    for (int64_t v = 0; v < n; ++v) {
+      dist[v] = -1;
+      sigma[v] = 0.0;
+      delta[v] = 0.0;
+    }
+    dist[s] = 0;
+    sigma[s] = 1.0;
+    int64_t head = 0, tail = 0; /* S doubles as the BFS queue: visit order */
+    S[tail++] = s;
+    while (head < tail) {
+      const int64_t v = S[head++];
+      for (int64_t k = row_ptr[v]; k < row_ptr[v + 1]; ++k) {
+        const int64_t w = col_idx[k];
+        if (dist[w] < 0) {
+          dist[w] = dist[v] + 1;
+          S[tail++] = w;
+        }
+        if (dist[w] == dist[v] + 1) sigma[w] += sigma[v];
+      }
+    }
+    /* reverse visit order: every successor of w is finished before w */
+    for (int64_t j = tail - 1; j >= 0; --j) {
+      const int64_t w = S[j];
+      for (int64_t k = row_ptr[w]; k < row_ptr[w + 1]; ++k) {
+        const int64_t v = col_idx[k];
+        if (dist[v] == dist[w] + 1) delta[w] += sigma[w] / sigma[v] * (1.0 + delta[v]);
+      }
+      if (w != s) bc[w] += delta[w];
+    }
+  }
+  free(S);
+  free(dist);
+  free(sigma);
+  free(delta);
+  return 0;
+}

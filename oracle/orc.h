@@ -42,6 +42,16 @@ int orc_sssp_dijkstra(int64_t n, const int64_t *row_ptr, const int32_t *col_idx,
 int orc_bfs(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t source,
             int32_t *level);
 
+/* Betweenness centrality (PAPER.md P5@8318-8911: "equal to the number of shortest paths
+ * from all nodes to all others that pass through that node"; two phases after [6]: a BFS
+ * shortest-path tree of the unweighted graph, then a backward pass over it).  Reading
+ * R10: Freeman/Brandes betweenness over ordered pairs of the given sources,
+ *   bc[v] = sum_{s in sources} sum_{t != s, t != v} sigma_st(v) / sigma_st
+ * computed by Brandes' recurrence delta_s(w) = sum_{v: w in P_s(v)} sigma_sw/sigma_sv (1 + delta_s(v)),
+ * sigma and delta in fp64.  All n vertices as sources = exact BC. */
+int orc_bc(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int64_t *sources,
+           int64_t n_sources, double *bc);
+
 #ifdef __cplusplus
 }
 #endif
