@@ -38,7 +38,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["inl", "reference"], default="inl")
-    ap.add_argument("--op", choices=["spmv", "sssp", "bfs", "pagerank"], default="spmv")
+    ap.add_argument("--op", choices=["spmv", "sssp", "bfs", "pagerank", "bc"], default="spmv")
     ap.add_argument("--scale", type=int, default=None, help="R-MAT scale at N=1 (default per op)")
     ap.add_argument("--edge-factor", type=int, default=16)
     ap.add_argument("--bins", type=str, default="", help="t_thread,t_warp,t_block,grid_chunk,cta")
@@ -50,7 +50,7 @@ def parse():
     return ap.parse_args()
 
 
-DEFAULT_SCALE = {"spmv": 22, "sssp": 23, "bfs": 23, "pagerank": 25}
+DEFAULT_SCALE = {"spmv": 22, "sssp": 23, "bfs": 23, "pagerank": 25, "bc": 20}
 
 
 def peaks():
@@ -137,7 +137,8 @@ def cpu_cores():
 def build_workload(op, scale, ef, world, rank, torch):
     import inlgen
     from paper_conf_icpp_liwb15_b200 import inl
-    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC}[op]
+    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC,
+             "bc": inlgen.SYMMETRIC}[op]
     n = 1 << scale
     b = inl.partition_rows(n, world)
     g = inlgen.dev_build(scale, ef, seed=inlgen.SEED_GRAPH, flags=flags, row_begin=b[rank], row_end=b[rank + 1])
@@ -222,6 +223,7 @@ def run_inl(a):
             dist.broadcast(src_t, 0)
             srcs = [int(v) for v in src_t.tolist() if v >= 0]
         out_arr = torch.empty(A.n_global, dtype=torch.int32, device="cuda")
+        bc_arr = torch.empty(A.n_global, dtype=torch.float64, device="cuda") if a.op == "bc" else None
         state = {"i": 0, "last": None}
 
         def step():
@@ -229,6 +231,8 @@ def run_inl(a):
             state["i"] += 1
             if a.op == "sssp":
                 state["last"] = inl.sssp(ctx, A, W["w"], s, out_arr, plan)
+            elif a.op == "bc":  # one source per step: forward BFS DAG + backward dependencies
+                state["last"] = inl.bc(ctx, A, [s], bc_arr, plan)
             else:
                 state["last"] = inl.bfs(ctx, A, s, out_arr, plan)
         units_local = None
@@ -244,6 +248,7 @@ def run_inl(a):
     reached = []
     # the dominant kernel(s), timed live by the library with events on its own stream
     kernels = (["k_gather", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
+               else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
                else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_sssp_split"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
@@ -253,7 +258,7 @@ def run_inl(a):
         ev0.record(stream)
         for _ in range(a.steps):
             step()
-            if a.op in ("sssp", "bfs"):
+            if a.op in ("sssp", "bfs", "bc"):
                 reached.append(state["last"])
         ev1.record(stream)
         torch.cuda.synchronize()
@@ -278,7 +283,7 @@ def run_inl(a):
         ms = float(t.item())
     ms_step = ms / a.steps
 
-    if a.op in ("sssp", "bfs"):
+    if a.op in ("sssp", "bfs", "bc"):
         # m_reached = sum of degrees of reached vertices (directed CSR entries) per source
         tot_edges = 0
         for i in range(a.steps):
@@ -293,8 +298,15 @@ def run_inl(a):
             lo = g["row_begin"]
             tot_edges += int(deg[reached_mask[lo:lo + A.n_rows]].sum().item())
         units_local = tot_edges
-        relax = sum(r["edges_relaxed"] for r in reached)
-        bytes_local = 8 * relax + 16 * sum(r["frontier_total"] for r in reached)
+        if a.op == "bc":
+            # every reached edge is scanned twice (forward, backward): col + level per scan;
+            # per reached vertex: row_ptr twice, sigma, delta, bc, queue
+            bytes_local = 16 * tot_edges + 64 * sum(r["frontier_total"] for r in reached)
+            for r in reached:
+                r["edges_relaxed"] = 2 * tot_edges // max(len(reached), 1)
+        else:
+            relax = sum(r["edges_relaxed"] for r in reached)
+            bytes_local = 8 * relax + 16 * sum(r["frontier_total"] for r in reached)
         if all(r.get("launches", 0) > 0 for r in reached):  # counted by the library
             launches_per_step = sum(r["launches"] for r in reached) / len(reached)
         else:
@@ -324,7 +336,8 @@ def run_inl(a):
             "data": "synthetic (R-MAT A,B,C=.57,.19,.19, Philox seeds graph=1 val=3 x=4 w=2, generated on GPU)",
             "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
                                     "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
-                                    "bfs": "cfg5 BFS R-MAT symmetric"}[a.op],
+                                    "bfs": "cfg5 BFS R-MAT symmetric",
+                                    "bc": "NEXT-3 betweenness R-MAT symmetric (one source per step)"}[a.op],
                        "op": a.op, "scale": scale, "edge_factor": a.edge_factor, "n": A.n_global,
                        "nnz_total": units_total // a.steps // (a.iterations if a.op == "pagerank" else 1) if a.op in ("spmv", "pagerank") else None,
                        "rows_per_gpu": A.n_rows, "parallelism": f"row-blocks x{world}",
@@ -347,7 +360,7 @@ def run_inl(a):
         e2e = e2e_spmv(a, ctx, g, W, torch, world, rank)
         if rank == 0:
             out["e2e"] = e2e
-    if a.op in ("sssp", "bfs") and rank == 0:
+    if a.op in ("sssp", "bfs", "bc") and rank == 0:
         out["config"]["sources"] = srcs
         out["config"]["iterations"] = [r["iterations"] for r in reached]
         out["config"]["relaxations_per_m_reached"] = round(sum(r["edges_relaxed"] for r in reached) / max(units_total, 1), 3)
@@ -437,6 +450,8 @@ def cpu_baseline(op, g, W, a, torch, budget_s=10.0):
     else:
         d = oracle.bfs(rp, ci, src)
         reached = d >= 0
+        if op == "bc":
+            oracle.bc(rp, ci, [src])
     dt = time.perf_counter() - t0
     m = int((rp[1:] - rp[:-1])[reached].sum())
     return {"value": round(m / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
@@ -460,7 +475,8 @@ def run_reference(a):
         have_gpu = torch.cuda.is_available()
     except Exception:
         have_gpu = False
-    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC}[a.op]
+    flags = {"spmv": 0, "pagerank": inlgen.TRANSPOSE, "sssp": inlgen.SYMMETRIC, "bfs": inlgen.SYMMETRIC,
+             "bc": inlgen.SYMMETRIC}[a.op]
     if have_gpu:
         g = inlgen.dev_build(scale, a.edge_factor, seed=inlgen.SEED_GRAPH, flags=flags)
         rp, ci = g["row_ptr"].cpu().numpy(), g["col_idx"].cpu().numpy()
@@ -485,6 +501,8 @@ def run_reference(a):
         fn = (lambda: oracle.sssp(rp, ci, wts, src)) if a.op == "sssp" else (lambda: oracle.bfs(rp, ci, src))
         d = fn()
         reached = (d != 0xFFFFFFFF) if a.op == "sssp" else (d >= 0)
+        if a.op == "bc":
+            fn = lambda: oracle.bc(rp, ci, [src])  # noqa: E731
         units = int(np.diff(rp)[reached].sum())
         sample = f"one full {a.op} from source {src} per step"
     for _ in range(max(a.warmup, 0)):
@@ -500,7 +518,8 @@ def run_reference(a):
             "data": "synthetic (same R-MAT recipe and seeds as the inl arm)",
             "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
                                     "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
-                                    "bfs": "cfg5 BFS R-MAT symmetric"}[a.op],
+                                    "bfs": "cfg5 BFS R-MAT symmetric",
+                                    "bc": "NEXT-3 betweenness R-MAT symmetric (one source per step)"}[a.op],
                        "op": a.op, "scale": scale, "edge_factor": a.edge_factor, "n": int(n), "nnz_total": int(len(ci))},
             "cpu_baseline": {"value": round(v, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": round(v, 5), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

@@ -174,6 +174,16 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
                    inl_stats *stats, inl_plan plan);
 
+/* Betweenness centrality (P5@8318-8911; reading R10 of DESIGN.md): for each of the
+ * n_sources vertices in `sources` (a HOST array of global ids), a BFS shortest-path DAG
+ * with path counts sigma, then Brandes' backward dependency sweep;
+ *   bc[v] = sum_{s in sources} sum_{t != s, v} sigma_st(v) / sigma_st      (fp64)
+ * bc [n_global] double (device or host), overwritten.  All vertices as sources = exact
+ * BC (ordered pairs; an undirected graph's usual value is half).  One GPU (no row
+ * blocks).  stats: iterations = forward levels over all sources.  Blocks until done. */
+inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t n_sources, double *bc,
+                  inl_stats *stats, inl_plan plan);
+
 /* Kernel timer (measurement only; off by default).  While enabled, every launch of the
  * path's main kernels ("k_gather", "k_gather_thread_only", "k_expand_flat",
  * "k_expand_grid", "k_bfs_bottom_up") is bracketed by CUDA events recorded on the ctx

@@ -589,4 +589,25 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
   });
 }
 
+inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t n_sources, double *bc,
+                  inl_stats *stats, inl_plan plan) {
+  if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
+  return guarded(ctx, [&] {
+    check_csr(G);
+    INL_CHECK(n_sources >= 0 && (n_sources == 0 || sources != nullptr), "sources is NULL");
+    INL_CHECK(n_sources == 0 || !is_device(sources), "sources must be a host array");
+    for (int64_t i = 0; i < n_sources; ++i)
+      INL_CHECK(sources[i] >= 0 && sources[i] < G->n_global, "source out of range");
+    INL_CHECK(G->n_global == 0 || bc != nullptr, "bc is NULL");
+    INL_CHECK(G->row_begin == 0 && G->n_rows == G->n_global, "bc: one GPU, full CSR (no row blocks)");
+    DeviceGuard g(ctx->device);
+    inl_csr d = device_csr(ctx, G);
+    if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
+    StagedOut<double> o = stage_out(ctx->h_y, bc, G->n_global);
+    bc_run(ctx, d, sources, n_sources, o.dev, stats);
+    finish_out(ctx, o);
+    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  });
+}
+
 }  // extern "C"

@@ -223,6 +223,9 @@ constexpr int kTemplateFlags = INL_BINS_TPL_DUAL_QUEUE | INL_BINS_TPL_DBUF_GLOBA
 bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *val, const float *x, float *y);
 // colblock.cu: builds `cb` for the column space `cols` (raw ids in [0, ncols), CSR order)
 void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool sort_rows = false);
+// bc.cu
+void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
+            inl_stats *stats);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);
 }  // namespace inl

@@ -92,6 +92,7 @@ def lib() -> C.CDLL:
         L.inl_pagerank.argtypes = [vp, C.POINTER(CsrT), vp, C.c_float, i32, vp, vp]
         L.inl_sssp.argtypes = [vp, C.POINTER(CsrT), vp, i64, vp, C.POINTER(StatsT), vp]
         L.inl_bfs.argtypes = [vp, C.POINTER(CsrT), i64, vp, C.POINTER(StatsT), vp]
+        L.inl_bc.argtypes = [vp, C.POINTER(CsrT), vp, i64, vp, C.POINTER(StatsT), vp]
         L.inl_ktimer_enable.argtypes = [vp, i32]
         L.inl_ktimer_read.argtypes = [vp, C.c_char_p, C.POINTER(i64), C.POINTER(C.c_double)]
         for f in ("inl_ctx_create", "inl_ctx_set_stream", "inl_ctx_destroy", "inl_partition_rows",
@@ -314,3 +315,17 @@ def bfs(ctx: Ctx, G: Csr, source: int, level, plan: Plan | None = None) -> dict:
                          _plan_handle(plan)), ctx)
     return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total,
             "launches": st.launches, "host_syncs": st.host_syncs}
+
+
+def bc(ctx: Ctx, G: Csr, sources, out, plan: Plan | None = None) -> dict:
+    """Betweenness centrality over `sources` (PAPER.md P5@8318; reading R10): out[n_global]
+    float64 (torch CUDA tensor or numpy), overwritten; blocks until done."""
+    import numpy as np
+    ctx.sync_stream()
+    s = G.struct()
+    src = np.ascontiguousarray(np.asarray(sources, dtype=np.int64))
+    st = StatsT()
+    _check(lib().inl_bc(ctx.handle, C.byref(s), src.ctypes.data if src.size else None, len(src), _ptr(out),
+                        C.byref(st), _plan_handle(plan)), ctx)
+    return {"iterations": st.iterations, "frontier_total": st.frontier_total, "launches": st.launches,
+            "host_syncs": st.host_syncs}

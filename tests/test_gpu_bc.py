@@ -1,0 +1,97 @@
+"""GPU parity: inl_bc (CUDA through the C-ABI) vs oracle.bc (Brandes, fp64 CPU).
+
+Bar: fp64 on both sides; the sums differ only in order (thread-serial rows follow the
+oracle's order, warp / CTA rows use fixed trees), so max relative error <= 1e-9 and
+vertices of zero betweenness exactly 0.  Path counts are integers (exact in fp64).
+"""
+import numpy as np
+import pytest
+import torch
+
+import inlgen
+import oracle
+from graphs import csr_from_edges
+from paper_conf_icpp_liwb15_b200 import inl
+
+pytestmark = pytest.mark.gpu
+RTOL = 1e-9
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    return inl.Ctx(0)
+
+
+def gpu_bc(ctx, rp, ci, n, sources):
+    out = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+    st = inl.bc(ctx, inl.Csr(dev(rp), dev(ci), n), sources, out)
+    return out.cpu().numpy(), st
+
+
+def check(got, ref):
+    z = ref == 0
+    assert np.all(got[z] == 0), "zero betweenness must be exactly 0"
+    if (~z).any():
+        assert np.max(np.abs(got[~z] - ref[~z]) / ref[~z]) <= RTOL
+
+
+def test_closed_forms(ctx):
+    n = 40
+    rp, ci, _ = csr_from_edges(n, [(i, i + 1) for i in range(n - 1)], symmetric=True)
+    got, _ = gpu_bc(ctx, rp, ci, n, range(n))
+    assert np.array_equal(got, [2.0 * i * (n - 1 - i) for i in range(n)])
+    k = 5000  # hub above the warp bin: CTA-mapped (global delayed buffer) in both phases
+    rp, ci, _ = csr_from_edges(k + 1, [(0, i) for i in range(1, k + 1)], symmetric=True)
+    got, _ = gpu_bc(ctx, rp, ci, k + 1, range(0, k + 1, 7))
+    ref = oracle.bc(rp, ci, range(0, k + 1, 7))
+    check(got, ref)
+    assert got[0] == ref[0]  # integer-valued for a star
+    n = 30
+    rp, ci, _ = csr_from_edges(n, [(i, j) for i in range(n) for j in range(i + 1, n)], symmetric=True)
+    assert np.all(gpu_bc(ctx, rp, ci, n, range(n))[0] == 0)
+
+
+def test_cfg1_exact_all_sources(ctx):
+    g = inlgen.host_build(12, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    got, st = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, range(g.n_global))
+    check(got, oracle.bc(g.row_ptr, g.col_idx))
+    assert st["iterations"] >= g.n_global
+
+
+def test_directed_and_repeatable(ctx):
+    g = inlgen.host_build(13, 16, seed=inlgen.SEED_GRAPH)  # directed R-MAT
+    srcs = inlgen.sources(g.row_ptr, 16)
+    got, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
+    check(got, oracle.bc(g.row_ptr, g.col_idx, srcs))
+    again, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
+    assert np.array_equal(got, again)
+
+
+def test_scale16_sources(ctx):
+    g = inlgen.host_build(16, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    srcs = inlgen.sources(g.row_ptr, 8)
+    got, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
+    check(got, oracle.bc(g.row_ptr, g.col_idx, srcs))
+
+
+def test_random_small_and_edge_cases(ctx):
+    rng = np.random.default_rng(3)
+    for trial in range(30):
+        n = int(rng.integers(1, 40))
+        e = [(int(rng.integers(n)), int(rng.integers(n))) for _ in range(int(rng.integers(0, 4 * n)))]
+        rp, ci, _ = csr_from_edges(n, e, symmetric=bool(trial % 2))
+        srcs = sorted(set(int(v) for v in rng.integers(0, n, size=5)))
+        got, _ = gpu_bc(ctx, rp, ci, n, srcs)
+        check(got, oracle.bc(rp, ci, srcs))
+    rp, ci, _ = csr_from_edges(4, [(1, 2)], symmetric=True)
+    got, _ = gpu_bc(ctx, rp, ci, 4, [])  # no sources: zeros
+    assert np.all(got == 0)
+    out = np.full(4, np.nan)  # host output buffer
+    inl.bc(ctx, inl.Csr(rp, ci, 4), [0, 1], out)
+    assert np.all(out == 0)
+    with pytest.raises(RuntimeError):
+        gpu_bc(ctx, rp, ci, 4, [4])
