@@ -116,6 +116,8 @@ typedef struct {
   int64_t cb_nnz;         /* their nonzeros */
   int64_t cb_width;       /* column-block width K (x floats held in shared memory) */
   int64_t cb_threshold;   /* rows of degree > cb_threshold are column-blocked */
+  int64_t symmetric;      /* 1: every edge's reverse is present (full square CSR with sorted rows);
+                             enables BFS bottom-up and BC pull steps for calls using this plan */
 } inl_plan_info;
 
 const char *inl_version(void);
@@ -169,7 +171,8 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
 inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source,
                     uint32_t *dist, inl_stats *stats, inl_plan plan);
 
-/* BFS (P5@11591): level-synchronous frontier expansion; level [n_global] int32,
+/* BFS (P5@11591): level-synchronous frontier expansion (direction-optimizing when the
+ * plan found the graph symmetric); level [n_global] int32,
  * -1 = unreachable, level[source] = 0 (replicated).  Blocks until converged. */
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
                    inl_stats *stats, inl_plan plan);

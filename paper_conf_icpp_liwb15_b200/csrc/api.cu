@@ -583,7 +583,7 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
     StagedOut<int32_t> o = stage_out(ctx->h_y, level, G->n_global);
     Bins b = plan ? plan->bins : resolve_bins(nullptr);
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
-    bfs_run(ctx, d, b, source, o.dev, stats);
+    bfs_run(ctx, d, b, source, o.dev, stats, plan && plan->symmetric);
     finish_out(ctx, o);
     INL_CUDA(cudaStreamSynchronize(ctx->stream));
   });
@@ -604,7 +604,7 @@ inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t
     inl_csr d = device_csr(ctx, G);
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
     StagedOut<double> o = stage_out(ctx->h_y, bc, G->n_global);
-    bc_run(ctx, d, sources, n_sources, o.dev, stats);
+    bc_run(ctx, d, sources, n_sources, o.dev, stats, plan && plan->symmetric);
     finish_out(ctx, o);
     INL_CUDA(cudaStreamSynchronize(ctx->stream));
   });

@@ -4,9 +4,9 @@
 // delta (Brandes' recurrence) into bc.  Both phases are the paper's irregular nested loop
 // (outer: the vertices of one level, inner: their adjacency), load-balanced with its
 // templates: a CTA takes 256 level vertices; degree <= kBcThread runs serially in one
-// thread, larger ones are deferred to a shared-memory buffer and run warp-mapped
-// (dbuf-shared, P5@3623), the largest go to a global buffer that a second kernel runs
-// CTA-mapped (dbuf-global, P5@2721).
+// thread, larger ones are deferred to shared-memory buffers and run by 8-lane groups
+// (<= kBcGroup) or warps (dbuf-shared, P5@3623), the largest are cut into pieces in a
+// global buffer that a second kernel runs CTA-mapped (dbuf-global, P5@2721).
 //   forward  (level L):  v unvisited -> claimed for L+1 (atomicCAS), enqueued; every edge
 //                        into level L+1 adds sigma[u] to sigma[v] (fp64 atomicAdd: path
 //                        counts are integers, exact below 2^53).
@@ -14,6 +14,7 @@
 //                        (pull, no atomics; fixed order per vertex), bc[w] += delta[w].
 #include <cooperative_groups.h>
 
+#include <cstdlib>
 #include <vector>
 
 #include "inl_internal.cuh"
@@ -25,9 +26,10 @@ namespace inl {
 namespace {
 
 constexpr int kBcNT = 256;
-constexpr int kBcThread = 16;    // degree <= 16: one thread (thread-mapped inner loop)
-constexpr int kBcWarp = 4096;    // degree <= 4096: one warp; above: kBcChunk-edge pieces, one CTA each
-constexpr int kBcChunk = 4096;   // (global buffer; backward pieces combined in piece order)
+constexpr int kBcThread = 2;     // degree <= 2: one thread (thread-mapped inner loop)
+constexpr int kBcGroup = 64;     // degree <= 64: 8 lanes (a quarter warp)
+constexpr int kBcWarp = 256;     // degree <= 256: one warp; above: kBcChunk-edge pieces, one CTA each
+constexpr int kBcChunk = 2048;   // (global buffer; backward pieces combined in piece order)
 
 struct BcArgs {
   const int64_t *rp;
@@ -77,10 +79,10 @@ __device__ __forceinline__ void bwd_finish(const BcArgs &a, int32_t w, double d)
 
 template <bool FWD>
 __global__ void __launch_bounds__(kBcNT) k_bc_level(BcArgs a) {
-  __shared__ int32_t wl[kBcNT];
-  __shared__ int nw;
+  __shared__ int32_t wl[kBcNT], gl[kBcNT];
+  __shared__ int nw, ng;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) nw = 0;
+  if (tid == 0) nw = ng = 0;
   __syncthreads();
   const int i = a.lo + blockIdx.x * kBcNT + tid;
   if (i < a.hi) {
@@ -96,6 +98,8 @@ __global__ void __launch_bounds__(kBcNT) k_bc_level(BcArgs a) {
         for (int64_t k = rs; k < re; ++k) d += bwd_term(a, sw, __ldg(a.col + k));
         bwd_finish(a, u, d);
       }
+    } else if (re - rs <= kBcGroup) {
+      gl[atomicAdd(&ng, 1)] = u;
     } else if (re - rs <= kBcWarp) {
       wl[atomicAdd(&nw, 1)] = u;
     } else {
@@ -106,6 +110,26 @@ __global__ void __launch_bounds__(kBcNT) k_bc_level(BcArgs a) {
     }
   }
   __syncthreads();
+  // 8-lane groups (4 vertices per warp per round; warp-uniform round count)
+  const int sub = lane & 7, grp = lane >> 3;
+  for (int j0 = warp * 4; j0 < ng; j0 += kBcNT / 8) {
+    const int j = j0 + grp;
+    double d = 0.0;
+    int32_t u = -1;
+    if (j < ng) {
+      u = gl[j];
+      const int64_t rs = a.rp[u], re = a.rp[u + 1];
+      const double su = a.sigma[u];
+      for (int64_t k = rs + sub; k < re; k += 8) {
+        if (FWD) fwd_edge(a, su, __ldg(a.col + k));
+        else d += bwd_term(a, su, __ldg(a.col + k));
+      }
+    }
+    if (!FWD) {
+      for (int o = 4; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+      if (sub == 0 && u >= 0) bwd_finish(a, u, d);
+    }
+  }
   for (int j = warp; j < nw; j += kBcNT / 32) {  // warp-mapped (shared delayed buffer)
     const int32_t u = wl[j];
     const int64_t rs = a.rp[u], re = a.rp[u + 1];
@@ -165,6 +189,25 @@ __global__ void k_bc_combine(BcArgs a) {
   }
 }
 
+// Forward step pulled from the unvisited side (direction optimisation, Beamer et al.,
+// SC'12) for large frontiers of a symmetric graph (rows list the predecessors): an unvisited v sums sigma over ALL its level-L neighbours
+// (plain loads, no atomics, neighbour order); a non-zero sum puts v on level L+1.
+__global__ void __launch_bounds__(kBcNT) k_bc_pull(BcArgs a, int64_t n) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    if (a.level[v] != -1) continue;
+    double s = 0.0;
+    for (int64_t k = a.rp[v]; k < a.rp[v + 1]; ++k) {
+      const int32_t u = __ldg(a.col + k);
+      if (a.level[u] == a.L) s += a.sigma[u];
+    }
+    if (s > 0.0) {
+      a.level[v] = a.L + 1;
+      a.sigma[v] = s;
+      enqueue(a.Q, a.hi, a.qcount, (int32_t)v);
+    }
+  }
+}
+
 __global__ void k_bc_init(int32_t *level, double *sigma, int64_t n, int64_t s, int32_t *Q) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
     level[v] = v == s ? 0 : -1;
@@ -187,7 +230,7 @@ int grid_of(int64_t n, int sms) {
 }  // namespace
 
 void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
-            inl_stats *stats) {
+            inl_stats *stats, bool symmetric) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   INL_CHECK(n < INT32_MAX, "bc: n must be < 2^31");
@@ -206,6 +249,11 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
   INL_CUDA(cudaGetLastError());
   int64_t launches = 1, syncs = 0, iters = 0, ftotal = 0;
   std::vector<int> off;
+  static int pull_div = -1;  // pull when the frontier holds more than n / pull_div vertices
+  if (pull_div < 0) {
+    pull_div = 8;  // measured: 16 -> 4.92 ms, 8 -> 4.14 ms, 64 -> 4.31 ms per scale-22 source
+    if (const char *e = getenv("INL_BC_PULL_DIV")) pull_div = atoi(e);  // 0: never pull
+  }
   for (int64_t si = 0; si < n_sources; ++si) {
     const int64_t s = sources[si];
     k_bc_init<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(level, sigma, n, s, Q);
@@ -219,12 +267,16 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
       a.L = L;
       if (a.hi == a.lo) break;
       INL_CUDA(cudaMemsetAsync(cnt, 0, 3 * sizeof(int), st));
-      {
+      if (symmetric && pull_div > 0 && (int64_t)(a.hi - a.lo) * pull_div > n) {  // large frontier: pull
+        KScope ks(ctx, "k_bc_fwd");
+        k_bc_pull<<<ctx->num_sms * 8, kBcNT, 0, st>>>(a, n);
+        launches += 1;
+      } else {
         KScope ks(ctx, "k_bc_fwd");
         k_bc_level<true><<<(a.hi - a.lo + kBcNT - 1) / kBcNT, kBcNT, 0, st>>>(a);
         k_bc_big<true><<<ctx->num_sms * 4, kBcNT, 0, st>>>(a);
+        launches += 2;
       }
-      launches += 2;
       INL_CUDA(cudaGetLastError());
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, cnt, sizeof(int), cudaMemcpyDeviceToHost, st));
       INL_CUDA(cudaStreamSynchronize(st));

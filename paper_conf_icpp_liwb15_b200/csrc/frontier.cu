@@ -928,7 +928,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
 }
 
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
-             inl_stats *stats) {
+             inl_stats *stats, bool symmetric) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
@@ -952,7 +952,9 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   uint32_t *fa = nullptr, *fb = nullptr;
   bool bu = false;       // direction of the previous step
   bool queue_ok = true;  // f.F holds the frontier (else the bitmap fa does)
-  const bool allow_bu = !(b.flags & INL_BINS_THREAD_ONLY) && n >= 4096;
+  // bottom-up scans a vertex's row for frontier parents: valid only when rows list the
+  // predecessors too (a symmetric graph, verified by the plan)
+  const bool allow_bu = symmetric && !(b.flags & INL_BINS_THREAD_ONLY) && n >= 4096;
   if (allow_bu) {
     fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
     fb = fa + nwords + 1;

@@ -182,6 +182,7 @@ struct inl_plan_s {
   inl::DevBuf pr_col;          // int32 [nnz]: gather columns in the compact space (hot kept)
   inl::DevBuf pr_hot;          // int32 [pr_nhot]: hot slots in the compact space
   int64_t pr_nhot = 0;         // PageRank's hot slots (a prefix of the plan's)
+  bool symmetric = false;  // every edge's reverse is present (checked at plan time, sorted rows)
   // column-blocked long rows: SpMV (the CSR's column space) and PageRank (compact space)
   inl::CbPlan cb, pr_cb;
 };
@@ -216,8 +217,10 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
 // frontier.cu
 void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
               uint32_t *dist, inl_stats *st);
+// symmetric: the plan verified that every edge (u, v) has its reverse (v, u), so a vertex's
+// row lists its predecessors too (bottom-up / pull steps are valid)
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
-             inl_stats *st);
+             inl_stats *st, bool symmetric);
 // templates.cu: the paper's dual-queue / dbuf-global / dbuf-shared SpMV (false: no template flag)
 constexpr int kTemplateFlags = INL_BINS_TPL_DUAL_QUEUE | INL_BINS_TPL_DBUF_GLOBAL | INL_BINS_TPL_DBUF_SHARED;
 bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *val, const float *x, float *y);
@@ -225,7 +228,7 @@ bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *va
 void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool sort_rows = false);
 // bc.cu
 void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
-            inl_stats *stats);
+            inl_stats *stats, bool symmetric);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);
 }  // namespace inl

@@ -188,6 +188,35 @@ __global__ void k_bin_stats(const int64_t *__restrict__ rp, int64_t n, Bins b,
   }
 }
 
+// symmetry check: every entry (r, c) of a square CSR has (c, r) — binary search of r in row
+// c (rows sorted; an unsorted row just fails the check, which only disables bottom-up)
+__global__ void k_check_symmetric(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n,
+                                  int *__restrict__ bad) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n;
+       r += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    bool ok = true;
+    for (int64_t k = rp[r] + lane; k < rp[r + 1]; k += 32) {
+      const int32_t c = col[k];
+      if (c < 0 || c >= n) {
+        ok = false;
+        break;
+      }
+      int64_t lo = rp[c], hi = rp[c + 1];
+      while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (col[mid] < r) lo = mid + 1;
+        else hi = mid;
+      }
+      if (lo >= rp[c + 1] || col[lo] != r) {
+        ok = false;
+        break;
+      }
+    }
+    if (__any_sync(0xffffffffu, !ok) && lane == 0) atomicExch(bad, 1);
+  }
+}
+
 int grid_for(int64_t n, int num_sms) {
   int64_t g = (n + 255) / 256;
   const int64_t cap = (int64_t)num_sms * 16;
@@ -342,6 +371,18 @@ void build_plan(inl_plan p) {
     INL_CUDA(cudaGetLastError());
   }
   build_hot_remap(p);
+  p->symmetric = false;
+  if (p->n_rows == p->n_global && p->row_begin == 0) {
+    int *bad = (int *)ctx->s_f.get(64);
+    INL_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), st));
+    k_check_symmetric<<<grid_for(n * 32, ctx->num_sms), 256, 0, st>>>(p->row_ptr, p->col_idx, n, bad);
+    INL_CUDA(cudaGetLastError());
+    int h_bad = 1;
+    INL_CUDA(cudaMemcpyAsync(&h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    p->symmetric = h_bad == 0;
+  }
+  p->info.symmetric = p->symmetric ? 1 : 0;
   cb_build(p, p->cb, p->col_idx, p->n_global);
   p->pr_cb.active = false;
   INL_CUDA(cudaMemsetAsync(p->ticket.get(16), 0, 16, st));

@@ -58,7 +58,7 @@ class PlanInfoT(C.Structure):
                 ("nnz_warp", C.c_int64), ("nnz_block", C.c_int64), ("nnz_grid", C.c_int64),
                 ("n_grid_chunks", C.c_int64), ("bins", BinsT), ("cb_rows", C.c_int64),
                 ("cb_runs", C.c_int64), ("cb_nnz", C.c_int64), ("cb_width", C.c_int64),
-                ("cb_threshold", C.c_int64)]
+                ("cb_threshold", C.c_int64), ("symmetric", C.c_int64)]
 
 
 _lib = None

@@ -95,3 +95,25 @@ def test_random_small_and_edge_cases(ctx):
     assert np.all(out == 0)
     with pytest.raises(RuntimeError):
         gpu_bc(ctx, rp, ci, 4, [4])
+
+
+def test_pull_steps_with_symmetric_plan(ctx):
+    """With a plan that verified symmetry, large frontiers are expanded by pull steps."""
+    g = inlgen.host_build(15, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    plan = inl.Plan(ctx, A)
+    assert plan.info()["symmetric"] == 1
+    srcs = inlgen.sources(g.row_ptr, 6)
+    out = torch.empty(g.n_global, dtype=torch.float64, device="cuda")
+    inl.bc(ctx, A, srcs, out, plan)
+    got = out.cpu().numpy()
+    check(got, oracle.bc(g.row_ptr, g.col_idx, srcs))
+    plain, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)  # push-only path
+    check(got, plain)
+    d = inlgen.host_build(13, 16, seed=inlgen.SEED_GRAPH)  # directed: plan must not pull
+    Ad = inl.Csr(dev(d.row_ptr), dev(d.col_idx), d.n_global)
+    pd = inl.Plan(ctx, Ad)
+    out = torch.empty(d.n_global, dtype=torch.float64, device="cuda")
+    s = inlgen.sources(d.row_ptr, 4)
+    inl.bc(ctx, Ad, s, out, pd)
+    check(out.cpu().numpy(), oracle.bc(d.row_ptr, d.col_idx, s))

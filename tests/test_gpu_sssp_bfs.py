@@ -137,3 +137,18 @@ def test_scale18_certificate_all_sources(ctx):
         if i < 2:
             assert np.array_equal(dh, oracle.sssp(rph, cih, wh, s))
             assert np.array_equal(lvh, oracle.bfs(rph, cih, s))
+
+
+def test_directed_graph_with_plan(ctx):
+    """Bottom-up BFS steps need rows to list predecessors: the plan enables them only for a
+    symmetric CSR; a directed R-MAT through a plan must still match the oracle."""
+    g = inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH)  # directed
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    plan = inl.Plan(ctx, A)
+    assert plan.info()["symmetric"] == 0
+    for s in inlgen.sources(g.row_ptr, 4):
+        lv = torch.zeros(g.n_global, dtype=torch.int32, device="cuda")
+        inl.bfs(ctx, A, s, lv, plan)
+        assert np.array_equal(lv.cpu().numpy(), oracle.bfs(g.row_ptr, g.col_idx, s))
+    gs = inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    assert inl.Plan(ctx, inl.Csr(dev(gs.row_ptr), dev(gs.col_idx), gs.n_global)).info()["symmetric"] == 1
