@@ -372,7 +372,7 @@ void build_plan(inl_plan p) {
   }
   build_hot_remap(p);
   p->symmetric = false;
-  if (p->n_rows == p->n_global && p->row_begin == 0) {
+  if (!p->transient && p->n_rows == p->n_global && p->row_begin == 0) {  // one-shot calls skip it
     int *bad = (int *)ctx->s_f.get(64);
     INL_CUDA(cudaMemsetAsync(bad, 0, sizeof(int), st));
     k_check_symmetric<<<grid_for(n * 32, ctx->num_sms), 256, 0, st>>>(p->row_ptr, p->col_idx, n, bad);

@@ -12,3 +12,5 @@ run --op bfs --steps 9 --warmup 3
 run --op bfs --steps 9 --warmup 3 --thread-only
 run --op pagerank --steps 3 --warmup 1
 run --op bfs --scale 26 --steps 4 --warmup 1
+run --op bc --steps 8 --warmup 3
+run --op bc --scale 22 --steps 4 --warmup 3
