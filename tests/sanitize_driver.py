@@ -35,6 +35,22 @@ def main():
     src = inlgen.sources(s.row_ptr, 1)[0]
     inl.sssp(ctx, As, w, src, d)
     inl.bfs(ctx, As, src, d)
+    ps = inl.Plan(ctx, As)  # symmetric plan: BFS bottom-up steps, BC pull steps
+    inl.bfs(ctx, As, src, d, ps)
+    inl.sssp(ctx, As, w, src, d, inl.Plan(ctx, As, inl.bins(flags=inl.BINS_SSSP_DEVLOOP)))
+    bc = torch.empty(s.n_global, dtype=torch.float64, device="cuda")
+    srcs = inlgen.sources(s.row_ptr, 3)
+    inl.bc(ctx, As, srcs, bc)
+    inl.bc(ctx, As, srcs, bc, ps)
+    # the paper's templates and the column-blocked bin (small blocks: several per row)
+    val, x = dev(inlgen.values_host(g.row_ptr, g.col_idx)), dev(inlgen.vector_host(g.n_global))
+    for fl in (inl.BINS_TPL_DUAL_QUEUE, inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DBUF_SHARED):
+        inl.spmv(ctx, A, val, x, y, inl.Plan(ctx, A, inl.bins(t_thread=16, t_warp=16, t_block=16, cta_threads=64,
+                                                               flags=fl)))
+    os.environ["INL_CB_K"] = "128"
+    os.environ["INL_CB_MULT"] = "1"
+    inl.spmv(ctx, A, val, x, y, inl.Plan(ctx, A, inl.bins(t_warp=16, flags=inl.BINS_COLBLOCK)))
+    inl.pagerank(ctx, At, dev(t.out_degree), r, 0.85, 3, inl.Plan(ctx, At, inl.bins(t_warp=16, flags=inl.BINS_COLBLOCK)))
     torch.cuda.synchronize()
     print("sanitize driver ok")
 
