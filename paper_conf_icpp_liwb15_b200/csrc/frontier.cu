@@ -146,6 +146,8 @@ struct BfsOp {
   int L;
   bool enqueue;      // !DIST
   uint64_t pol_stream;
+  const int64_t *rp = nullptr;       // !DIST: degree sum of the next frontier -> *mf
+  unsigned long long *mf = nullptr;  //   (Beamer's m_f, for the direction switch)
   __device__ __forceinline__ uint32_t load(int32_t) const { return 0u; }
   __device__ __forceinline__ void visit(int32_t v, int32_t *q, int *cnt) const {
     if (enqueue) {
@@ -153,6 +155,7 @@ struct BfsOp {
       const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
       if (!(old & bit)) {
         level[v] = L + 1;
+        if (mf) atomicAdd(mf, (unsigned long long)(rp[v + 1] - rp[v]));
         push(q, cnt, v);
       }
     } else {
@@ -192,6 +195,14 @@ struct BfsOp {
         won |= 1u << j;
         level[vv[j]] = L + 1;
       }
+    if (mf) {  // degree sum of the claimed vertices (one atomic per warp)
+      unsigned long long dsum = 0;
+#pragma unroll
+      for (int j = 0; j < K; ++j)
+        if ((won >> j) & 1u) dsum += (unsigned long long)(rp[vv[j] + 1] - rp[vv[j]]);
+      for (int o = 16; o > 0; o >>= 1) dsum += __shfl_xor_sync(0xffffffffu, dsum, o);
+      if ((threadIdx.x & 31) == 0 && dsum) atomicAdd(mf, dsum);
+    }
     push_batch(q, cnt, vv, won);
   }
 };
@@ -610,7 +621,7 @@ __global__ void k_bfs_apply(const uint8_t *__restrict__ next, int64_t n, int32_t
 __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t n,
                                 uint32_t *__restrict__ visited, const uint32_t *__restrict__ fcur,
                                 uint32_t *__restrict__ fnext, int32_t *__restrict__ level, int L,
-                                int *__restrict__ count) {
+                                int *__restrict__ count, unsigned long long *__restrict__ mf) {
   const int lane = threadIdx.x & 31;
   const int64_t nwords = (n + 31) / 32;
   for (int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; w < nwords;
@@ -618,6 +629,7 @@ __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *_
     const uint32_t vis = visited[w];
     const int64_t v = w * 32 + lane;
     bool found = false;
+    unsigned long long dg = 0;
     if (v < n && !((vis >> lane) & 1u)) {
       const int64_t e = rp[v + 1];
       for (int64_t k = rp[v]; k < e; ++k) {
@@ -627,8 +639,13 @@ __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *_
           break;
         }
       }
-      if (found) level[v] = L + 1;
+      if (found) {
+        level[v] = L + 1;
+        dg = (unsigned long long)(e - rp[v]);
+      }
     }
+    for (int o = 16; o > 0; o >>= 1) dg += __shfl_xor_sync(0xffffffffu, dg, o);
+    if (lane == 0 && dg) atomicAdd(mf, dg);
     const uint32_t nw = __ballot_sync(0xffffffffu, found);
     if (lane == 0) {
       fnext[w] = nw;
@@ -955,6 +972,17 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   // bottom-up scans a vertex's row for frontier parents: valid only when rows list the
   // predecessors too (a symmetric graph, verified by the plan)
   const bool allow_bu = symmetric && !(b.flags & INL_BINS_THREAD_ONLY) && n >= 4096;
+  // Beamer's m_f (degree sum of the next frontier) and m_u (edges of unvisited vertices)
+  unsigned long long *mfp = (unsigned long long *)(f.counts + 10);
+  unsigned long long mf_next = 0;
+  double m_u = (double)G.nnz;
+  auto read_level = [&](int *nf, unsigned long long *mfn) {
+    INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 48, cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    *nf = ((volatile int *)ctx->pinned)[0];
+    *mfn = *(volatile unsigned long long *)((int *)ctx->pinned + 10);
+    m_u -= (double)*mfn;
+  };
   if (allow_bu) {
     fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
     fb = fa + nwords + 1;
@@ -963,20 +991,23 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
     ftotal += nF;
     if (!DIST) {
       if (nF == 0) break;
-      const bool want_bu = allow_bu && (bu ? nF > n / 256 : nF > n / 24);
+      // Beamer's switch: enter bottom-up when the frontier's edges exceed the unvisited
+      // edges / 14 (or it holds > n/24 vertices), leave it below n/256 vertices
+      const bool want_bu = allow_bu && (bu ? nF > n / 256 : (nF > n / 24 || (double)mf_next * 14.0 > (double)m_u));
       if (want_bu) {
         if (queue_ok) {  // frontier queue -> bitmap
           INL_CUDA(cudaMemsetAsync(fa, 0, sizeof(uint32_t) * nwords, st));
           k_queue_to_bitmap<<<grid_for(nF, ctx->num_sms), 256, 0, st>>>(f.F, nF, fa);
         }
         INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+        INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
         {
           KScope ks(ctx, "k_bfs_bottom_up");
           k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
-                                                           f.counts);
+                                                           f.counts, mfp);
         }
         INL_CUDA(cudaGetLastError());
-        nF = read_count(ctx, f.counts);
+        read_level(&nF, &mf_next);
         std::swap(fa, fb);
         queue_ok = false;
       } else {
@@ -985,9 +1016,10 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           k_bitmap_to_queue<<<grid_for(nwords, ctx->num_sms), 256, 0, st>>>(fa, n, f.F, f.counts);
           INL_CUDA(cudaGetLastError());
         }
-        BfsOp op{bm, level, nullptr, n, L, true, 0};
+        BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, mfp};
+        INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
         expand(ctx, G, b, f, nF, op);
-        nF = read_count(ctx, f.counts);
+        read_level(&nF, &mf_next);
         std::swap(f.F, f.Fout);
         queue_ok = true;
       }
