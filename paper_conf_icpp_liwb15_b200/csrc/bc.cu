@@ -40,6 +40,7 @@ struct BcArgs {
   int lo, hi;       // this level's slice of Q
   int L;
   int *qcount;      // forward: vertices enqueued for level L+1 (at Q[hi + i])
+  unsigned long long *mf;  // forward: degree sum of the vertices enqueued for level L+1
   int2 *big;        // global buffer: (vertex, piece) of the largest-degree vertices
   int *bigcount;
   int4 *bigv;       // (vertex, first piece, pieces) per large vertex (backward combine)
@@ -48,12 +49,26 @@ struct BcArgs {
   int32_t source;
 };
 
-__device__ __forceinline__ void enqueue(int32_t *Q, int base, int *cnt, int32_t v) {
+// append v to level L+1 (one counter atomic per coalesced group)
+__device__ __forceinline__ void enqueue(const BcArgs &a, int32_t v) {
   cg::coalesced_group g = cg::coalesced_threads();
   int pos = 0;
-  if (g.thread_rank() == 0) pos = atomicAdd(cnt, (int)g.size());
+  if (g.thread_rank() == 0) pos = atomicAdd(a.qcount, (int)g.size());
   pos = g.shfl(pos, 0) + (int)g.thread_rank();
-  Q[base + pos] = v;
+  a.Q[a.hi + pos] = v;
+}
+
+// m_f of the level just built: degree sum of Q[hi, hi + *qcount) (Beamer's frontier edge
+// count for the push / pull choice), one atomic per warp
+__global__ void k_bc_degsum(BcArgs a) {
+  const int cntv = *(volatile int *)a.qcount;
+  unsigned long long s = 0;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < cntv; i += gridDim.x * blockDim.x) {
+    const int32_t v = a.Q[a.hi + i];
+    s += (unsigned long long)(a.rp[v + 1] - a.rp[v]);
+  }
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0 && s) atomicAdd(a.mf, s);
 }
 
 // forward edge (u at level L, sigma su) -> v
@@ -61,7 +76,7 @@ __device__ __forceinline__ void fwd_edge(const BcArgs &a, double su, int32_t v) 
   int lv = a.level[v];
   if (lv == -1) {
     const int old = atomicCAS(a.level + v, -1, a.L + 1);
-    if (old == -1) enqueue(a.Q, a.hi, a.qcount, v);
+    if (old == -1) enqueue(a, v);
     lv = a.L + 1;  // whoever won, only level L+1 is claimed in this step
   }
   if (lv == a.L + 1) atomicAdd(a.sigma + v, su);
@@ -203,7 +218,7 @@ __global__ void __launch_bounds__(kBcNT) k_bc_pull(BcArgs a, int64_t n) {
     if (s > 0.0) {
       a.level[v] = a.L + 1;
       a.sigma[v] = s;
-      enqueue(a.Q, a.hi, a.qcount, (int32_t)v);
+      enqueue(a, (int32_t)v);
     }
   }
 }
@@ -244,7 +259,8 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
   int2 *big = (int2 *)ctx->s_e.get(sizeof(int2) * maxp);
   double *bigpart = (double *)ctx->s_g.get(sizeof(double) * maxp);
   int4 *bigv = (int4 *)ctx->s_tmp.get(sizeof(int4) * (G.nnz / kBcWarp + 16));
-  int *cnt = (int *)ctx->s_f.get(64);
+  int *cnt = (int *)ctx->s_f.get(64);  // [0] queue [1] pieces [2] large vertices; m_f at byte 16
+  unsigned long long *mfp = (unsigned long long *)(cnt + 4);
   k_zero_d<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(bc, n);
   INL_CUDA(cudaGetLastError());
   int64_t launches = 1, syncs = 0, iters = 0, ftotal = 0;
@@ -254,20 +270,29 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
     pull_div = 8;  // measured: 16 -> 4.92 ms, 8 -> 4.14 ms, 64 -> 4.31 ms per scale-22 source
     if (const char *e = getenv("INL_BC_PULL_DIV")) pull_div = atoi(e);  // 0: never pull
   }
+  static double pull_edge = -1.0;  // > 0: pull when m_f * pull_edge > m_u (edge rule), else n/pull_div
+  if (pull_edge < 0.0) {
+    pull_edge = 0.5;  // measured on one box at scale 22: n/8 rule 5.38, 0.5 -> 4.16, 1 -> 4.34, 2 -> 5.64 ms
+    if (const char *e = getenv("INL_BC_PULL_EDGE")) pull_edge = atof(e);
+  }
   for (int64_t si = 0; si < n_sources; ++si) {
     const int64_t s = sources[si];
     k_bc_init<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(level, sigma, n, s, Q);
     ++launches;
     off.assign({0, 1});
-    BcArgs a{G.row_ptr, G.col_idx, level, sigma, delta, bc, Q, 0, 0, 0, cnt, big, cnt + 1, bigv, cnt + 2, bigpart,
-             (int32_t)s};
+    BcArgs a{G.row_ptr, G.col_idx, level, sigma, delta, bc, Q, 0, 0, 0, cnt, mfp, big, cnt + 1, bigv, cnt + 2,
+             bigpart, (int32_t)s};
+    double m_u = (double)G.nnz;       // edges of unvisited vertices (Beamer)
+    unsigned long long mf_next = 0;   // edges of the current frontier
     for (int L = 0;; ++L) {  // forward: one level per step
       a.lo = off[L];
       a.hi = off[L + 1];
       a.L = L;
       if (a.hi == a.lo) break;
-      INL_CUDA(cudaMemsetAsync(cnt, 0, 3 * sizeof(int), st));
-      if (symmetric && pull_div > 0 && (int64_t)(a.hi - a.lo) * pull_div > n) {  // large frontier: pull
+      INL_CUDA(cudaMemsetAsync(cnt, 0, 24, st));  // counters + m_f
+      const bool pull = symmetric && (pull_edge > 0.0 ? (double)mf_next * pull_edge > m_u
+                                                      : pull_div > 0 && (int64_t)(a.hi - a.lo) * pull_div > n);
+      if (pull) {  // large frontier: pull from the unvisited side
         KScope ks(ctx, "k_bc_fwd");
         k_bc_pull<<<ctx->num_sms * 8, kBcNT, 0, st>>>(a, n);
         launches += 1;
@@ -277,11 +302,17 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
         k_bc_big<true><<<ctx->num_sms * 4, kBcNT, 0, st>>>(a);
         launches += 2;
       }
+      if (pull_edge > 0.0) {
+        k_bc_degsum<<<ctx->num_sms * 2, 256, 0, st>>>(a);
+        ++launches;
+      }
       INL_CUDA(cudaGetLastError());
-      INL_CUDA(cudaMemcpyAsync(ctx->pinned, cnt, sizeof(int), cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, cnt, 24, cudaMemcpyDeviceToHost, st));
       INL_CUDA(cudaStreamSynchronize(st));
       ++syncs;
       off.push_back(a.hi + *(volatile int *)ctx->pinned);
+      mf_next = *(volatile unsigned long long *)((char *)ctx->pinned + 16);
+      m_u -= (double)mf_next;
       ++iters;
     }
     ftotal += off.back();
