@@ -632,12 +632,18 @@ __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *_
     unsigned long long dg = 0;
     if (v < n && !((vis >> lane) & 1u)) {
       const int64_t e = rp[v + 1];
-      for (int64_t k = rp[v]; k < e; ++k) {
-        const int32_t u = __ldg(col + k);
-        if ((__ldg(fcur + (u >> 5)) >> (u & 31)) & 1u) {
-          found = true;
-          break;
-        }
+      // 4 neighbours per step: their column loads, then their frontier-bit loads, are
+      // issued back to back (the scan is a chain of dependent loads otherwise)
+      for (int64_t k = rp[v]; k < e && !found; k += 4) {
+        int32_t u[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) u[j] = k + j < e ? __ldg(col + k + j) : -1;
+        uint32_t fw[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) fw[j] = u[j] >= 0 ? __ldg(fcur + (u[j] >> 5)) : 0u;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          if (u[j] >= 0 && ((fw[j] >> (u[j] & 31)) & 1u)) found = true;
       }
       if (found) {
         level[v] = L + 1;
