@@ -11,7 +11,9 @@
 //                        into level L+1 adds sigma[u] to sigma[v] (fp64 atomicAdd: path
 //                        counts are integers, exact below 2^53).
 //   backward (level L):  delta[w] = sum_{v in N(w), level[v] = L+1} sigma[w]/sigma[v] (1+delta[v])
-//                        (pull, no atomics; fixed order per vertex), bc[w] += delta[w].
+//                        (pull, no atomics; fixed order per vertex), bc[w] += delta[w]; a
+//                        finished w leaves (1+delta)/sigma, its level and the sweep's tag in
+//                        one 16-B record (one gather per backward edge).
 #include <cooperative_groups.h>
 
 #include <cstdlib>
@@ -31,6 +33,14 @@ constexpr int kBcGroup = 64;     // degree <= 64: 8 lanes (a quarter warp)
 constexpr int kBcWarp = 256;     // degree <= 256: one warp; above: kBcChunk-edge pieces, one CTA each
 constexpr int kBcChunk = 2048;   // (global buffer; backward pieces combined in piece order)
 
+// A finished vertex of the backward sweep: (1 + delta) / sigma, its level, and the tag
+// (source number + 1) of the sweep that wrote it — one 16-B gather per backward edge
+// instead of level + sigma + delta.
+struct __align__(16) BcPk {
+  double coef;
+  int32_t level, tag;
+};
+
 struct BcArgs {
   const int64_t *rp;
   const int32_t *col;
@@ -47,6 +57,8 @@ struct BcArgs {
   int *bigvcount;
   double *bigpart;  // backward partial sum per piece
   int32_t source;
+  BcPk *pk;
+  int32_t tag;
 };
 
 // append v to level L+1 (one counter atomic per coalesced group)
@@ -82,13 +94,18 @@ __device__ __forceinline__ void fwd_edge(const BcArgs &a, double su, int32_t v) 
   if (lv == a.L + 1) atomicAdd(a.sigma + v, su);
 }
 
-// backward term of edge w -> v
+// backward term of edge w -> v: sigma_w / sigma_v (1 + delta_v) for a successor v
 __device__ __forceinline__ double bwd_term(const BcArgs &a, double sw, int32_t v) {
-  return a.level[v] == a.L + 1 ? sw / a.sigma[v] * (1.0 + a.delta[v]) : 0.0;
+  const BcPk p = a.pk[v];
+  return p.tag == a.tag && p.level == a.L + 1 ? sw * p.coef : 0.0;
 }
 
 __device__ __forceinline__ void bwd_finish(const BcArgs &a, int32_t w, double d) {
-  a.delta[w] = d;
+  BcPk p;
+  p.coef = (1.0 + d) / a.sigma[w];
+  p.level = a.L;
+  p.tag = a.tag;
+  a.pk[w] = p;
   if (w != a.source) a.bc[w] += d;
 }
 
@@ -253,7 +270,9 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
   int32_t *level = (int32_t *)ctx->s_a.get(sizeof(int32_t) * n);
   int32_t *Q = (int32_t *)ctx->s_b.get(sizeof(int32_t) * (n + 1));
   double *sigma = (double *)ctx->s_c.get(sizeof(double) * n);
-  double *delta = (double *)ctx->s_d.get(sizeof(double) * n);
+  double *delta = nullptr;  // folded into pk
+  BcPk *pk = (BcPk *)ctx->s_d.get(sizeof(BcPk) * n);
+  INL_CUDA(cudaMemsetAsync(pk, 0, sizeof(BcPk) * n, st));  // tag 0 = never written
   // pieces of the vertices above kBcWarp: <= nnz / kBcChunk + (their number <= nnz / kBcWarp)
   const int64_t maxp = G.nnz / kBcChunk + G.nnz / kBcWarp + 16;
   int2 *big = (int2 *)ctx->s_e.get(sizeof(int2) * maxp);
@@ -281,7 +300,7 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
     ++launches;
     off.assign({0, 1});
     BcArgs a{G.row_ptr, G.col_idx, level, sigma, delta, bc, Q, 0, 0, 0, cnt, mfp, big, cnt + 1, bigv, cnt + 2,
-             bigpart, (int32_t)s};
+             bigpart, (int32_t)s, pk, (int32_t)(si + 1)};
     double m_u = (double)G.nnz;       // edges of unvisited vertices (Beamer)
     unsigned long long mf_next = 0;   // edges of the current frontier
     for (int L = 0;; ++L) {  // forward: one level per step
