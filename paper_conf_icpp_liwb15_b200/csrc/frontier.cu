@@ -1022,7 +1022,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           k_bitmap_to_queue<<<grid_for(nwords, ctx->num_sms), 256, 0, st>>>(fa, n, f.F, f.counts);
           INL_CUDA(cudaGetLastError());
         }
-        BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, mfp};
+        BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, allow_bu ? mfp : nullptr};  // m_f only when it decides
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
         expand(ctx, G, b, f, nF, op);
         read_level(&nF, &mf_next);
