@@ -727,8 +727,14 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
   INL_CUDA(cudaMemsetAsync(f.counts, 0, 2 * sizeof(int), st));
   ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
                f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
+  const int tpl = b.flags & kTemplateFlags;
+  INL_CHECK(tpl != INL_BINS_TPL_DUAL_QUEUE, "dual-queue template: SpMV only (SSSP/BFS: dbuf-shared, dbuf-global)");
+  if (tpl) {  // the paper's delayed-buffer templates (template study): lbTHRES = t_thread
+    a.t_warp = b.t_thread;  // no warp bin: above lbTHRES is block-mapped ...
+    a.t_block = tpl == INL_BINS_TPL_DBUF_SHARED ? INT32_MAX / 2 : b.t_thread;  // ... in smem / via the grid buffer
+  }
   if (nF > 0) {
-    if (b.flags & INL_BINS_THREAD_ONLY) {  // the paper's baseline: thread-mapped, no balancing
+    if ((b.flags & INL_BINS_THREAD_ONLY) || tpl) {  // the paper's baseline (thread-mapped) / templates
       KScope ks(ctx, "k_expand");
       k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
     } else {
@@ -853,7 +859,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   // source for the host-driven one (profiles/r01/sssp_devloop.txt) — its 4 launches per
   // step cost more than the ~40 host round trips they save
   const bool devloop = (b.flags & INL_BINS_SSSP_DEVLOOP) != 0;
-  if (!DIST && !(b.flags & INL_BINS_THREAD_ONLY) && devloop && sssp_delta() != 0xFFFFFFFFu && n > 0) {
+  if (!DIST && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && devloop && sssp_delta() != 0xFFFFFFFFu &&
+      n > 0) {
     sssp_run_dyn(ctx, G, b, w, source, dist, stats);
     return;
   }
@@ -879,7 +886,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
     farcnt = (int *)ctx->s_e.get(16);
     INL_CUDA(cudaMemsetAsync(farcnt, 0, 16, st));
     INL_CUDA(cudaMemsetAsync(keep, 0, sizeof(uint32_t) * nwb, st));
-    delta = b.flags & INL_BINS_THREAD_ONLY ? 0xFFFFFFFFu : sssp_delta();
+    // the baseline and the paper's templates run [5]'s plain frontier Bellman-Ford
+    delta = b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags) ? 0xFFFFFFFFu : sssp_delta();
     thr = delta;
   }
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(D, n, source);
@@ -977,7 +985,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   bool queue_ok = true;  // f.F holds the frontier (else the bitmap fa does)
   // bottom-up scans a vertex's row for frontier parents: valid only when rows list the
   // predecessors too (a symmetric graph, verified by the plan)
-  const bool allow_bu = symmetric && !(b.flags & INL_BINS_THREAD_ONLY) && n >= 4096;
+  const bool allow_bu = symmetric && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && n >= 4096;
   // Beamer's m_f (degree sum of the next frontier) and m_u (edges of unvisited vertices)
   unsigned long long *mfp = (unsigned long long *)(f.counts + 10);
   unsigned long long mf_next = 0;

@@ -79,3 +79,29 @@ def test_template_flags_are_spmv_only(ctx, g14):
     y = torch.empty(g14.n_rows, device="cuda")
     with pytest.raises(RuntimeError):
         inl.spmv(ctx, A, dev(np.ones(g14.nnz, np.float32)), dev(np.ones(g14.n_global, np.float32)), y, both)
+
+
+@pytest.mark.parametrize("name", ["dbuf_global", "dbuf_shared"])
+@pytest.mark.parametrize("lbt", [0, 8, 32, 1024])
+def test_frontier_templates_bit_exact(ctx, name, lbt):
+    """SSSP / BFS through the paper's delayed-buffer templates (plain frontier Bellman-Ford)."""
+    g = inlgen.host_build(12, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    w = inlgen.weights_host(g.row_ptr, g.col_idx)
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    plan = inl.Plan(ctx, A, inl.bins(t_thread=lbt if lbt > 0 else -1, t_warp=max(lbt, 16), t_block=max(lbt, 16),
+                                      flags=TPL[name]))
+    for s in inlgen.sources(g.row_ptr, 3):
+        d = torch.zeros(g.n_global, dtype=torch.int32, device="cuda")
+        inl.sssp(ctx, A, dev(w.view(np.int32)), s, d, plan)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(g.row_ptr, g.col_idx, w, s))
+        lv = torch.zeros(g.n_global, dtype=torch.int32, device="cuda")
+        inl.bfs(ctx, A, s, lv, plan)
+        assert np.array_equal(lv.cpu().numpy(), oracle.bfs(g.row_ptr, g.col_idx, s))
+
+
+def test_dual_queue_is_spmv_only_for_frontiers(ctx):
+    g = inlgen.host_build(10, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    lv = torch.zeros(g.n_global, dtype=torch.int32, device="cuda")
+    with pytest.raises(RuntimeError):
+        inl.bfs(ctx, A, 0, lv, inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DUAL_QUEUE)))
