@@ -25,6 +25,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--scale", type=int, default=23)
     ap.add_argument("--sources", type=int, default=3)
+    ap.add_argument("--only", type=str, default="", help="NAME[:LBT] — run one variant (for ncu)")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     stream = torch.cuda.Stream(0)
@@ -41,6 +42,9 @@ def main():
         for lbt in (32, 64, 128, 256, 1024):
             variants.append((name, dict(t_thread=lbt, t_warp=max(lbt, 16), t_block=max(lbt, 16), flags=fl), lbt))
     variants.append(("default (flat + grid, near-far)", dict(), None))
+    if a.only:
+        nm, _, lb = a.only.partition(":")
+        variants = [v for v in variants if v[0].startswith(nm) and (not lb or str(v[2]) == lb)]
     t1 = None
     for name, kw, lbt in variants:
         plan = inl.Plan(ctx, A, inl.bins(**kw))
