@@ -60,21 +60,35 @@ typedef struct {
 } inl_csr;
 
 /* Load-balancing thresholds (the paper's lbTHRES, P5@366; 0 = default).
- * A row / vertex of degree f goes to the
- *   thread bin  if f <= t_thread               (one lane runs the inner loop serially)
- *   warp bin    if t_thread < f <= t_warp       (one warp, lanes stride the inner loop)
- *   block bin   if t_warp < f <= t_block       (SpMV/PR: grid_chunk pieces, one warp each, for
- *                                                consecutive warps; SSSP/BFS: one CTA)
- *   grid bin    if f > t_block                 (grid_chunk-sized pieces spread over the grid)
- * Ties go to the lower bin (reading R6 of DESIGN.md: "f(i) greater than lbTHRES
- * is processed block-mapped", P11@1197).  t_thread = -1 means 0 (no thread bin).
+ *
+ * What each kernel family actually reads (a threshold not listed is ignored by it):
+ *  - DEFAULT fused kernels (no template flag).  The deferral threshold lbTHRES is t_warp:
+ *      SpMV / PageRank (k_gather): rows of degree <= t_warp form row tiles (one warp per
+ *        tile; inside a tile a row contained in one lane's 8 entries is summed serially by
+ *        that lane — thread-mapped — and a row crossing lanes by the warp's segmented scan
+ *        — warp-mapped; which of the two a row gets depends on its length and alignment,
+ *        not on t_thread); rows of degree > t_warp are cut into grid_chunk pieces, one warp
+ *        each, combined in piece order (the delayed buffer).  t_block only splits the
+ *        reported counts (rows_block / rows_grid); t_thread only splits rows_thread /
+ *        rows_warp in inl_plan_info.
+ *      SSSP / BFS (k_expand_flat, k_expand_grid): frontier vertices of degree <= t_warp are
+ *        buffered in shared memory and expanded CTA-wide, 8 edges per thread
+ *        (dbuf-shared); larger ones go to the global buffer as min(grid_chunk, 2048)-edge
+ *        pieces (dbuf-global).  t_thread and t_block are not read.
+ *  - The paper's templates (INL_BINS_TPL_*) and the T1 baseline: lbTHRES = t_thread, CTA =
+ *    cta_threads; the rows / vertices of degree > t_thread are block-mapped (SSSP/BFS
+ *    dbuf-global: through the global buffer in min(grid_chunk, 2048)-edge pieces).
+ * Ties go to the lower class (reading R6 of DESIGN.md: "f(i) greater than lbTHRES is
+ * processed block-mapped", P11@1197).  t_thread = -1 means 0.
  * flags: INL_BINS_THREAD_ONLY runs the paper's baseline (thread-mapped outer loop,
  * no load balancing, P5@14490).  INL_BINS_COLBLOCK (opt-in; measured slower at the
  * bench configs) processes SpMV/PR rows of degree > max(t_warp,
  * 4 * column blocks) column-blocked: a CTA holds one block of x in shared memory and
  * sums the row's entries in that block (one partial per (row, block) run, combined in
  * block order).  INL_BINS_SSSP_DEVLOOP (opt-in, one GPU): the SSSP near-far step loop
- * runs on the device, the host checks termination every few steps. */
+ * runs on the device, the host checks termination every few steps.  At most one
+ * INL_BINS_TPL_* flag, and none combined with another flag (else INL_ERR_INVALID_ARGUMENT
+ * from inl_plan_create). */
 enum {
   INL_BINS_THREAD_ONLY = 1,
   INL_BINS_COLBLOCK = 2,
@@ -90,10 +104,11 @@ enum {
   INL_BINS_TPL_DBUF_SHARED = 32
 };
 typedef struct {
-  int32_t t_thread;    /* default 8 */
-  int32_t t_warp;      /* default 128, in [16, 4096] (SpMV/PR warp tiles hold < 2*t_warp nnz) */
+  int32_t t_thread;    /* default 8; <= t_warp */
+  int32_t t_warp;      /* default 1024, in [16, 4096] (SpMV/PR tiles hold < 2048 + t_warp nnz) */
   int32_t t_block;     /* default 16384, >= t_warp */
-  int32_t grid_chunk;  /* default 8192 nnz per block/grid-bin piece (one warp each), in [32, 2^20] */
+  int32_t grid_chunk;  /* default 8192 nnz per SpMV/PR long-row piece (one warp each), in [32, 2^20];
+                          SSSP/BFS pieces are min(grid_chunk, 2048) edges */
   int32_t cta_threads; /* CTA size of the INL_BINS_TPL_* templates (multiple of 32 in [32, 1024],
                           default 256); the default kernels use fixed CTA shapes */
   int32_t flags;
@@ -109,7 +124,9 @@ typedef struct {
 
 /* Plan summary (for tests and the bench; counts per bin). */
 typedef struct {
-  int64_t n_tiles;        /* row tiles holding the thread/warp/block-bin rows */
+  int64_t n_tiles;        /* row tiles holding the rows of degree <= t_warp */
+  /* degree-class histogram by the thresholds (f <= t_thread, <= t_warp, <= t_block, above):
+     a diagnostic of the CSR's shape — see inl_bins for which classes a kernel maps differently */
   int64_t rows_thread, rows_warp, rows_block, rows_grid;
   int64_t nnz_thread, nnz_warp, nnz_block, nnz_grid;
   int64_t n_grid_chunks;  /* CTAs of the grid/long-row kernel */
@@ -153,9 +170,12 @@ inl_status inl_csr_validate(inl_ctx ctx, const inl_csr *A);
 
 /* SpMV (P5@10072, P5@10497): y[i] = sum_{k in row i} val[k] * x[col_idx[k]] for the
  * n_rows local rows; x has n_global entries.  fp32 in, fp32 accumulate, fp32 out.
- * Each row's reduction order depends only on its degree and the bins, so y is
- * bit-identical across partitions and runs.  plan: NULL = transient bins built
- * inside the call (cost included), else a plan created from this same inl_csr. */
+ * Deterministic: bit-identical run to run for the same CSR, bins and partition.  Across
+ * row-block partitions a row's fp32 summation order can differ (lane groups are aligned to
+ * the local work item), so y agrees within fp32 rounding, and bit-exactly when every partial
+ * sum is exactly representable (integer-valued data; reading R11).  plan: NULL =
+ * transient bins built inside the call (cost included), else a plan created from this
+ * same inl_csr. */
 inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y,
                     inl_plan plan);
 

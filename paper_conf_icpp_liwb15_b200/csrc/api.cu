@@ -103,6 +103,12 @@ Bins resolve_bins(const inl_bins *b) {
             "bins: need t_thread <= t_warp <= t_block");
   INL_CHECK(r.t_warp >= 16 && r.t_warp <= 4096, "bins.t_warp must be in [16, 4096]");
   INL_CHECK(r.grid_chunk >= 32 && r.grid_chunk <= (1 << 20), "bins.grid_chunk must be in [32, 2^20]");
+  const int tpl = r.flags & kTemplateFlags;
+  INL_CHECK((tpl & (tpl - 1)) == 0, "bins.flags: at most one paper template (INL_BINS_TPL_*)");
+  INL_CHECK(!(tpl && (r.flags & (INL_BINS_THREAD_ONLY | INL_BINS_COLBLOCK | INL_BINS_SSSP_DEVLOOP))),
+            "bins.flags: a paper template (INL_BINS_TPL_*) cannot be combined with other flags");
+  INL_CHECK(!((r.flags & INL_BINS_THREAD_ONLY) && (r.flags & (INL_BINS_COLBLOCK | INL_BINS_SSSP_DEVLOOP))),
+            "bins.flags: INL_BINS_THREAD_ONLY cannot be combined with other flags");
   if (r.flags & INL_BINS_THREAD_ONLY) {
     r.t_thread = r.t_warp = r.t_block = INT32_MAX / 2;
   }
@@ -199,7 +205,7 @@ bool same_csr(inl_plan p, const inl_csr &A) {
 }
 
 // plan (user or transient) for a device CSR
-inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user, inl_plan *transient_holder) {
+inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user) {
   if (user) {
     INL_CHECK(user->ctx == ctx, "plan belongs to another ctx");
     INL_CHECK(same_csr(user, A), "plan was created for a different CSR (pointers or sizes differ)");
@@ -208,7 +214,6 @@ inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user, inl_plan *transi
   // the ctx keeps one transient plan whose buffers are reused across calls
   if (!ctx->tplan) ctx->tplan = new inl_plan_s();
   inl_plan p = ctx->tplan;
-  (void)transient_holder;
   p->ctx = ctx;
   p->transient = true;
   p->n_rows = A.n_rows;
@@ -221,10 +226,6 @@ inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user, inl_plan *transi
   build_plan(p);
   return p;
 }
-
-struct PlanHolder {  // transient plans now live in the ctx (ctx->tplan); kept for clarity
-  inl_plan p = nullptr;
-};
 
 inl_status fail(inl_ctx ctx, inl_status code, const std::string &msg) {
   if (ctx) ctx->last_error = msg;
@@ -509,10 +510,7 @@ inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float
       INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
       spmv_template(ctx, d, plan->bins, dval, dx, yo.dev);
     } else {
-      PlanHolder tmp;
-      inl_plan p = get_plan(ctx, d, plan, &tmp.p);
-      spmv_run(ctx, p, dval, dx, yo.dev);
-      if (tmp.p) INL_CUDA(cudaStreamSynchronize(ctx->stream));  // transient plan freed on return
+      spmv_run(ctx, get_plan(ctx, d, plan), dval, dx, yo.dev);
     }
     finish_out(ctx, yo);
   });
@@ -539,10 +537,7 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
       raise(INL_ERR_UNSUPPORTED, "thread-only baseline plans are SpMV/SSSP/BFS only");
     if (plan && (plan->bins.flags & kTemplateFlags))
       raise(INL_ERR_UNSUPPORTED, "paper-template plans (INL_BINS_TPL_*) are SpMV only");
-    PlanHolder tmp;
-    inl_plan p = get_plan(ctx, d, plan, &tmp.p);
-    pagerank_run(ctx, p, dod, damping, iterations, ro.dev);
-    if (tmp.p) INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    pagerank_run(ctx, get_plan(ctx, d, plan), dod, damping, iterations, ro.dev);
     finish_out(ctx, ro);
   });
 }

@@ -154,10 +154,11 @@ template <bool VALS, class Epi>
 void launch_cb(inl_ctx ctx, const CbPlan &cb, const float *val, const float *x, const Epi &epi, double *dpart) {
   const CbArgs a = cb_args(cb);
   const size_t smem = (size_t)cb.K * 4;
-  static size_t configured = 0;  // per instantiation
-  if (smem > configured) {
+  static size_t configured[kMaxDevices] = {};  // per instantiation AND device
+  size_t &cf = configured[ctx->device % kMaxDevices];
+  if (smem > cf) {
     INL_CUDA(cudaFuncSetAttribute(k_cb<VALS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = smem;
+    cf = smem;
   }
   {
     KScope ks(ctx, "k_cb");

@@ -18,7 +18,9 @@
 //     BFS allreduce-max of an n-byte next-frontier map, each with a
 //     trailing termination word.
 #include <cooperative_groups.h>
+#include <algorithm>
 #include <cstdio>
+#include <string>
 #include <cstdlib>
 
 #include <cub/block/block_scan.cuh>
@@ -238,8 +240,10 @@ struct ExpandArgs {
   const int64_t *rp;
   const int32_t *col;
   int t_thread, t_warp, t_block, chunk;
-  int2 *gitems;  // grid-bin chunk buffer
+  int2 *gitems;  // grid-bin chunk buffer [gcap]
   int *gcount;
+  int gcap;      // its capacity (frontier_cfg: an upper bound of what one expansion emits)
+  int *oflow;    // set if an expansion ever needed more (-> INL_ERR_INTERNAL; never expected)
   int32_t *Fout;
   int *fcount;
   unsigned long long *relaxed;
@@ -287,6 +291,19 @@ __device__ __forceinline__ bool dyn_bind<SsspOp>(ExpandArgs &a, SsspOp &op, uint
   return true;
 }
 
+// Append the ceil(d / chunk) pieces of frontier vertex u to the grid buffer.  The buffer
+// holds gcap pieces, an upper bound of one expansion's output (frontier_cfg); a write past
+// it is dropped and flagged instead (the host turns the flag into INL_ERR_INTERNAL).
+__device__ __forceinline__ void emit_pieces(const ExpandArgs &a, int32_t u, int64_t d) {
+  const int nch = (int)((d + a.chunk - 1) / a.chunk);
+  const int base = atomicAdd(a.gcount, nch);
+  if (base + nch > a.gcap) {
+    atomicOr(a.oflow, 1);
+    return;
+  }
+  for (int c = 0; c < nch; ++c) a.gitems[base + c] = make_int2(u, c);
+}
+
 template <class Op>
 __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
@@ -314,9 +331,7 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
     } else if (d <= a.t_block) {
       lb[atomicAdd(&nb, 1)] = u;
     } else {  // grid bin: global delayed buffer
-      const int nch = (int)((d + a.chunk - 1) / a.chunk);
-      const int base = atomicAdd(a.gcount, nch);
-      for (int c = 0; c < nch; ++c) a.gitems[base + c] = make_int2(u, c);
+      emit_pieces(a, u, d);
     }
   }
   __syncthreads();
@@ -386,9 +401,7 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
     mydeg += (unsigned long long)dd;
     su = op.load(u);
     if (dd > a.t_warp) {  // grid bin: global delayed buffer
-      const int nch = (int)((dd + a.chunk - 1) / a.chunk);
-      const int base = atomicAdd(a.gcount, nch);
-      for (int c = 0; c < nch; ++c) a.gitems[base + c] = make_int2(u, c);
+      emit_pieces(a, u, dd);
     } else {
       d = (int)dd;
     }
@@ -468,7 +481,7 @@ __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
   __shared__ int n_s;  // one L2 read per CTA (every thread reading it would hit one L2 slice)
-  if (threadIdx.x == 0) n_s = __ldcg(a.gcount);
+  if (threadIdx.x == 0) n_s = min(__ldcg(a.gcount), a.gcap);  // dropped pieces were flagged
   __syncthreads();
   const int n = n_s;
   for (int it = blockIdx.x; it < n; it += gridDim.x) {
@@ -702,39 +715,70 @@ uint32_t sssp_delta() {
 struct FrontierBufs {
   int32_t *F, *Fout;
   int2 *gitems;
-  int *counts;  // [0] fcount [1] gcount
+  int64_t gcap;
+  int *counts;  // [0] fcount [1] gcount [2] grid-buffer overflow flag; u64 at [8] relaxed, [10] m_f
   unsigned long long *relaxed;
   int *h_counts;  // pinned
 };
+
+// Thresholds the expansion kernels use, and the grid-buffer capacity they imply.
+//  * default: k_expand_flat defers vertices of degree > t_warp to the grid buffer;
+//  * the paper's templates / the T1 baseline: k_expand (lbTHRES = t_thread; dbuf-global sends
+//    everything above it to the grid buffer, dbuf-shared and T1 nothing).
+// A frontier holds each vertex at most once, and a vertex of degree d > T emits ceil(d / C)
+// <= d / C + 1 pieces, so one expansion emits at most nnz / C + min(n_rows, nnz / (T + 1)).
+struct ExpandCfg {
+  int t_thread, t_warp, t_block, chunk;
+  bool flat;     // k_expand_flat (else k_expand)
+  int64_t gcap;  // grid-buffer capacity in pieces
+};
+
+ExpandCfg expand_cfg(const inl_csr &G, const Bins &b) {
+  ExpandCfg c{b.t_thread, b.t_warp, b.t_block, std::min(b.grid_chunk, 2048), true, 0};
+  const int tpl = b.flags & kTemplateFlags;
+  INL_CHECK(tpl != INL_BINS_TPL_DUAL_QUEUE, "dual-queue template: SpMV only (SSSP/BFS: dbuf-shared, dbuf-global)");
+  if (tpl) {  // the paper's delayed-buffer templates (template study): lbTHRES = t_thread
+    c.t_warp = b.t_thread;  // no warp bin: above lbTHRES is block-mapped ...
+    c.t_block = tpl == INL_BINS_TPL_DBUF_SHARED ? INT32_MAX / 2 : b.t_thread;  // ... in smem / via the grid buffer
+  }
+  c.flat = !((b.flags & INL_BINS_THREAD_ONLY) || tpl);
+  const int64_t T = c.flat ? c.t_warp : c.t_block;
+  c.gcap = G.nnz / c.chunk + std::min<int64_t>(G.n_rows, G.nnz / (T + 1)) + 64;
+  INL_CHECK(c.gcap < INT32_MAX, "frontier: grid buffer capacity exceeds 2^31 pieces");
+  return c;
+}
 
 FrontierBufs frontier_bufs(inl_ctx ctx, const inl_csr &G, const Bins &b) {
   FrontierBufs f;
   const int64_t n = G.n_global;
   f.F = (int32_t *)ctx->s_a.get(sizeof(int32_t) * (n + 1));
   f.Fout = (int32_t *)ctx->s_b.get(sizeof(int32_t) * (n + 1));
-  const int64_t mn = b.t_block < b.grid_chunk ? b.t_block : b.grid_chunk;
-  const int64_t gcap = G.nnz / (mn > 0 ? mn : 1) * 2 + 64;
-  f.gitems = (int2 *)ctx->s_c.get(sizeof(int2) * gcap);
+  f.gcap = expand_cfg(G, b).gcap;
+  f.gitems = (int2 *)ctx->s_c.get(sizeof(int2) * f.gcap);
   f.counts = (int *)ctx->s_f.get(64);
   f.relaxed = (unsigned long long *)(f.counts + 8);
   f.h_counts = (int *)ctx->pinned;
+  INL_CUDA(cudaMemsetAsync(f.counts, 0, 64, ctx->stream));
   return f;
+}
+
+// The grid-buffer overflow flag (never expected: gcap is an upper bound) -> INL_ERR_INTERNAL.
+void check_overflow(inl_ctx ctx, const FrontierBufs &f) {
+  int h = 0;
+  INL_CUDA(cudaMemcpyAsync(&h, f.counts + 2, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
+  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  if (h) raise(INL_ERR_INTERNAL, "frontier grid buffer overflow (capacity " + std::to_string(f.gcap) + " pieces)");
 }
 
 template <class Op>
 void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int nF, const Op &op) {
   cudaStream_t st = ctx->stream;
   INL_CUDA(cudaMemsetAsync(f.counts, 0, 2 * sizeof(int), st));
-  ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
-               f.gitems, f.counts + 1, f.Fout, f.counts, f.relaxed};
-  const int tpl = b.flags & kTemplateFlags;
-  INL_CHECK(tpl != INL_BINS_TPL_DUAL_QUEUE, "dual-queue template: SpMV only (SSSP/BFS: dbuf-shared, dbuf-global)");
-  if (tpl) {  // the paper's delayed-buffer templates (template study): lbTHRES = t_thread
-    a.t_warp = b.t_thread;  // no warp bin: above lbTHRES is block-mapped ...
-    a.t_block = tpl == INL_BINS_TPL_DBUF_SHARED ? INT32_MAX / 2 : b.t_thread;  // ... in smem / via the grid buffer
-  }
+  const ExpandCfg c = expand_cfg(G, b);
+  ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, c.t_thread, c.t_warp, c.t_block, c.chunk,
+               f.gitems, f.counts + 1, (int)f.gcap, f.counts + 2, f.Fout, f.counts, f.relaxed};
   if (nF > 0) {
-    if ((b.flags & INL_BINS_THREAD_ONLY) || tpl) {  // the paper's baseline (thread-mapped) / templates
+    if (!c.flat) {  // the paper's baseline (thread-mapped) / templates
       KScope ks(ctx, "k_expand");
       k_expand<Op><<<(nF + NT - 1) / NT, NT, 0, st>>>(a, op);
     } else {
@@ -756,6 +800,7 @@ int read_count(inl_ctx ctx, const int *d) {
 }
 
 void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_t ftotal) {
+  check_overflow(ctx, f);
   if (!st) return;
   unsigned long long r = 0;
   INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, ctx->stream));
@@ -800,8 +845,9 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(dist, n, source);
   INL_CUDA(cudaGetLastError());
-  ExpandArgs a{f.F, 0, G.row_ptr, G.col_idx, b.t_thread, b.t_warp, b.t_block, min(b.grid_chunk, 2048),
-               f.gitems, nullptr, f.Fout, nullptr, f.relaxed};
+  const ExpandCfg c = expand_cfg(G, b);
+  ExpandArgs a{f.F, 0, G.row_ptr, G.col_idx, c.t_thread, c.t_warp, c.t_block, c.chunk,
+               f.gitems, nullptr, (int)f.gcap, f.counts + 2, f.Fout, nullptr, f.relaxed};
   a.dyn = dy;
   SsspOp op{dist, w, nullptr, nullptr, 0, 0, true, 0, 0, nullptr, nullptr, nullptr};
   static int gmul = -1;  // grid multipliers (env INL_SSSP_GRIDS=split,flat,grid for tuning)
@@ -838,6 +884,7 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
     if (((volatile SsspDev *)hs)->done) break;
     if (batch < 16) batch *= 2;
   }
+  check_overflow(ctx, f);
   if (stats) {
     unsigned long long r = 0;
     INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, st));

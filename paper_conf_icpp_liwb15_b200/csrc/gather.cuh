@@ -28,9 +28,11 @@
 //    warp; the last chunk of a row (atomic ticket) combines the partials in chunk
 //    order (fp64).  Chunked rows of degree <= t_block are the BLOCK bin (their
 //    pieces go to consecutive warps), longer ones the GRID bin.
-//  * Each row's summation order depends only on its degree and the bins — never on
-//    the tile it lands in or on alignment — so results are bit-identical across
-//    partitions (multi-GPU) and runs.  No float atomics.
+//  * No float atomics: results are bit-identical run to run.  A row's summation order
+//    depends on where its entries fall in the 8-entry lane groups and 256-entry passes of
+//    its work item (aligned to the item's start), so a different row-block partition can
+//    round fp32 sums differently (within the fp32 bound; integer-valued data stays exact).
+//    DESIGN.md §3 reading R11.
 #pragma once
 #include <cuda/atomic>
 
@@ -449,10 +451,11 @@ template <int E, bool VALS, class Epi, int NWARP = 256 / E>
 void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
   const size_t smem = (size_t)gp.n_hot * 4 + 16;  // xs[0] is read (then discarded) by cold gathers
   auto kern = k_gather<E, VALS, Epi, NWARP>;
-  static size_t configured = 0;  // per instantiation
-  if (smem > configured) {
+  static size_t configured[kMaxDevices] = {};  // per instantiation AND device (the attribute is per device)
+  size_t &cf = configured[ctx->device % kMaxDevices];
+  if (smem > cf) {
     INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    configured = smem;
+    cf = smem;
   }
   int64_t grid = ctx->num_sms;
   const int64_t need = (gp.n_items + NWARP - 1) / NWARP;
@@ -502,7 +505,6 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     // each launch advances the counter by exactly n_items (successful grabs + one failing
     // grab per active warp), so the next launch's base is known on the host: no reset
     gp.base = p->ticket_base;
-    p->ticket_base += (unsigned long long)n_items;
     build_xhot(ctx, p, a.x, hot_over, n_hot);
     a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
     static int w24 = -1;
@@ -510,6 +512,7 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi);
     else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi);
     else launch_gather_t<8, VALS>(ctx, gp, a, epi);
+    p->ticket_base += (unsigned long long)n_items;  // only once the launch was accepted
   }
   if (use_cb) launch_cb<VALS>(ctx, *cb, a_in.val, a_in.x, epi, dpart ? dpart + n_items : nullptr);
 }

@@ -12,6 +12,7 @@
 namespace inl {
 
 constexpr int kTileRows = 256;  // max rows per SpMV/PR warp tile
+constexpr int kMaxDevices = 64;  // per-device caches of kernel attributes
 
 // One unit of work of the fused gather kernel (one warp): a tile (j < 0: rows [r0, r1),
 // all of degree <= t_warp, nonzeros [s, e), tile index t into the plan's non-empty-row

@@ -245,16 +245,6 @@ class Plan:
         d["bins"] = {f: getattr(i.bins, f) for f, _ in BinsT._fields_}
         return d
 
-    def ktimer_enable(self, on: bool = True) -> None:
-        """Bracket the main kernels' launches with CUDA events (measurement only)."""
-        _check(lib().inl_ktimer_enable(self.handle, 1 if on else 0), self)
-
-    def ktimer_read(self, kernel: str) -> tuple[int, float]:
-        """(launches, summed device ms) of `kernel` since ktimer_enable (syncs the stream)."""
-        n, ms = C.c_int64(), C.c_double()
-        _check(lib().inl_ktimer_read(self.handle, kernel.encode(), C.byref(n), C.byref(ms)), self)
-        return int(n.value), float(ms.value)
-
     def close(self) -> None:
         if getattr(self, "handle", None):
             lib().inl_plan_destroy(self.handle)

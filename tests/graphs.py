@@ -92,3 +92,27 @@ def certify_bfs(rp, ci, s, level):
     lv = np.asarray(level, np.int64)
     d = np.where(lv < 0, 0xFFFFFFFF, lv).astype(np.uint32)
     return certify_sssp(rp, ci, np.ones(len(ci), np.uint32), s, d)
+
+
+def csr_np(n, u, v, symmetric=True):
+    """Vectorised CSR build (sorted rows, no self-loops, duplicates merged) from edge arrays;
+    symmetric adds (v, u).  For large adversarial graphs where csr_from_edges is too slow."""
+    u = np.asarray(u, np.int64)
+    v = np.asarray(v, np.int64)
+    keep = u != v
+    u, v = u[keep], v[keep]
+    if symmetric:
+        u, v = np.concatenate([u, v]), np.concatenate([v, u])
+    key = np.unique(u * n + v)
+    rows, cols = key // n, key % n
+    rp = np.zeros(n + 1, np.int64)
+    np.add.at(rp, rows + 1, 1)
+    return np.cumsum(rp), cols.astype(np.int32)
+
+
+def pair_weights(rp, ci):
+    """Symmetric weights 1..255 keyed by the unordered pair (test-side recipe)."""
+    n = len(rp) - 1
+    src = np.repeat(np.arange(n, dtype=np.int64), np.diff(rp))
+    a, b = np.minimum(src, ci), np.maximum(src, ci)
+    return ((a * 2654435761 + b * 40503) % 255 + 1).astype(np.uint32)

@@ -7,6 +7,7 @@ import torch
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
 import inlgen  # noqa: E402
 from paper_conf_icpp_liwb15_b200 import inl  # noqa: E402
 
@@ -55,6 +56,21 @@ def main():
     os.environ["INL_CB_MULT"] = "1"
     inl.spmv(ctx, A, val, x, y, inl.Plan(ctx, A, inl.bins(t_warp=16, flags=inl.BINS_COLBLOCK)))
     inl.pagerank(ctx, At, dev(t.out_degree), r, 0.85, 3, inl.Plan(ctx, At, inl.bins(t_warp=16, flags=inl.BINS_COLBLOCK)))
+    # grid-bin buffer at its worst case: every vertex just above t_warp, fresh ctx, no plan;
+    # and dbuf-global with lbTHRES = 32 and the default t_block
+    from graphs import csr_np
+    rng = np.random.default_rng(3)
+    nb = 2400
+    brp, bci = csr_np(nb, np.repeat(np.arange(nb), 560), rng.integers(0, nb, nb * 560))
+    Ab = inl.Csr(dev(brp), dev(bci), nb)
+    wb = dev(inlgen.weights_host(brp, bci).view(np.int32))
+    db = torch.empty(nb, dtype=torch.int32, device="cuda")
+    c2 = inl.Ctx(0)
+    inl.bfs(c2, Ab, 0, db)
+    inl.sssp(c2, Ab, wb, 0, db)
+    pg = inl.Plan(c2, Ab, inl.bins(t_thread=32, flags=inl.BINS_TPL_DBUF_GLOBAL))
+    inl.bfs(c2, Ab, 0, db, pg)
+    inl.sssp(c2, Ab, wb, 0, db, pg)
     torch.cuda.synchronize()
     print("sanitize driver ok")
 

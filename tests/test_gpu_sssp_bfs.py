@@ -152,3 +152,61 @@ def test_directed_graph_with_plan(ctx):
         assert np.array_equal(lv.cpu().numpy(), oracle.bfs(g.row_ptr, g.col_idx, s))
     gs = inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
     assert inl.Plan(ctx, inl.Csr(dev(gs.row_ptr), dev(gs.col_idx), gs.n_global)).info()["symmetric"] == 1
+
+
+# ---- adversarial shapes for the grid-bin (dbuf-global) buffer (ADVICE high) ----
+def _dense_band_graph(n=20000, picks=700, seed=11):
+    """Every vertex of degree ~1025..2048: each one just above t_warp = 1024, so a frontier of
+    them emits one grid piece per ~1.1K edges (the worst case of the capacity bound)."""
+    from graphs import csr_np
+    rng = np.random.default_rng(seed)
+    u = np.repeat(np.arange(n), picks)
+    v = rng.integers(0, n, n * picks)
+    return csr_np(n, u, v)
+
+
+def test_grid_buffer_dense_band_fresh_ctx_no_plan():
+    from graphs import pair_weights
+    rp, ci = _dense_band_graph()
+    deg = np.diff(rp)
+    assert np.mean((deg > 1024) & (deg <= 2048)) > 0.95
+    w = pair_weights(rp, ci)
+    c = inl.Ctx(0)  # fresh ctx: nothing pre-grown by an earlier plan
+    for s in (0, 17, 19999):
+        d, _ = gpu_sssp(c, rp, ci, w, len(rp) - 1, s)
+        assert np.array_equal(d, oracle.sssp(rp, ci, w, s))
+        lv, _ = gpu_bfs(c, rp, ci, len(rp) - 1, s)
+        assert np.array_equal(lv, oracle.bfs(rp, ci, s))
+
+
+def test_grid_buffer_complete_bipartite_no_plan():
+    from graphs import csr_np, pair_weights
+    k = 1100
+    a = np.repeat(np.arange(k), k)
+    b = np.tile(np.arange(k, 2 * k), k)
+    rp, ci = csr_np(2 * k, a, b)
+    w = pair_weights(rp, ci)
+    c = inl.Ctx(0)
+    for s in (0, k, 2 * k - 1):
+        lv, _ = gpu_bfs(c, rp, ci, 2 * k, s)
+        assert np.array_equal(lv, oracle.bfs(rp, ci, s))
+        d, _ = gpu_sssp(c, rp, ci, w, 2 * k, s)
+        assert np.array_equal(d, oracle.sssp(rp, ci, w, s))
+
+
+@pytest.mark.parametrize("lbt", [8, 32])
+def test_dbuf_global_template_default_t_block(ctx, lbt):
+    """INL_BINS_TPL_DBUF_GLOBAL with lbTHRES = t_thread and the DEFAULT t_block: every vertex
+    above lbTHRES goes to the global buffer (inl.h documents this path)."""
+    g = inlgen.host_build(16, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    w = inlgen.weights_host(g.row_ptr, g.col_idx)
+    b = inl.bins(t_thread=lbt, flags=inl.BINS_TPL_DBUF_GLOBAL)
+    for s in inlgen.sources(g.row_ptr, 3):
+        d, _ = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, b)
+        assert np.array_equal(d, oracle.sssp(g.row_ptr, g.col_idx, w, s))
+        lv, _ = gpu_bfs(ctx, g.row_ptr, g.col_idx, g.n_global, s, b)
+        assert np.array_equal(lv, oracle.bfs(g.row_ptr, g.col_idx, s))
+    rp, ci = _dense_band_graph(n=4000, picks=600)
+    wb = inlgen.weights_host(rp, ci)
+    d, _ = gpu_sssp(ctx, rp, ci, wb, len(rp) - 1, 0, b)
+    assert np.array_equal(d, oracle.sssp(rp, ci, wb, 0))

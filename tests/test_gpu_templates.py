@@ -75,10 +75,11 @@ def test_template_flags_are_spmv_only(ctx, g14):
     r = torch.empty(g14.n_global, device="cuda")
     with pytest.raises(RuntimeError):
         inl.pagerank(ctx, A, dev(np.ones(g14.n_global, np.int32)), r, 0.85, 2, plan)
-    both = inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DUAL_QUEUE))
-    y = torch.empty(g14.n_rows, device="cuda")
-    with pytest.raises(RuntimeError):
-        inl.spmv(ctx, A, dev(np.ones(g14.nnz, np.float32)), dev(np.ones(g14.n_global, np.float32)), y, both)
+    # more than one template, or a template with another flag: rejected when the plan is made
+    for fl in (inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DUAL_QUEUE, inl.BINS_TPL_DUAL_QUEUE | inl.BINS_TPL_DBUF_GLOBAL,
+               inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DBUF_GLOBAL | inl.BINS_THREAD_ONLY):
+        with pytest.raises(RuntimeError):
+            inl.Plan(ctx, A, inl.bins(flags=fl))
 
 
 @pytest.mark.parametrize("name", ["dbuf_global", "dbuf_shared"])
