@@ -155,9 +155,26 @@ inl_status inl_ctx_destroy(inl_ctx ctx);
 inl_status inl_partition_rows(int64_t n, int32_t nranks, int64_t *bounds);
 
 /* NCCL bootstrap: rank 0 calls inl_nccl_unique_id and broadcasts the 128 bytes
- * (torch.distributed in the Python binding); every rank then calls inl_comm_init. */
+ * (torch.distributed in the Python binding); every rank then calls inl_comm_init.
+ * Once a ctx has a communicator it is one rank of a row-block job: its CSR is
+ * the row block [rank*B, rank*B + n_rows), B = ceil(n_global / nranks), and the ops run the
+ * exchange of SURVEY §8a row a12 (PageRank allgather, SSSP allreduce-min, BFS
+ * allreduce-max; inl_spmv_allgather).  nranks = 1 is allowed (the same code path). */
 inl_status inl_nccl_unique_id(uint8_t out[128]);
 inl_status inl_comm_init(inl_ctx ctx, const uint8_t uid[128], int32_t nranks, int32_t rank);
+
+/* Loopback communicator (tests and single-GPU studies of the multi-GPU path): P row-block
+ * contexts on ONE device exchange through the same calls as NCCL ranks, with device copies
+ * and a reduction kernel.  inl_loop_create makes a host object for nranks ranks; each rank's
+ * ctx (its own stream) joins it with inl_comm_init_loopback, and each rank must be driven by
+ * its own host thread, every rank calling the same ops in the same order (the NCCL rule):
+ * collectives block their host thread until all ranks reach them.  A rank whose call fails
+ * aborts the group, so its peers fail with INL_ERR_NCCL instead of hanging (also after a
+ * 300 s barrier timeout).  The group lives until it is destroyed AND every member ctx is. */
+typedef struct inl_loop_s *inl_loop;
+inl_status inl_loop_create(int32_t nranks, inl_loop *out);  /* nranks in [1, 64] */
+inl_status inl_loop_destroy(inl_loop group);
+inl_status inl_comm_init_loopback(inl_ctx ctx, inl_loop group, int32_t rank);
 
 /* Degree binning, built once and reused across calls on the
  * same CSR (device pointers only).  bins may be NULL (defaults). */
@@ -178,6 +195,14 @@ inl_status inl_csr_validate(inl_ctx ctx, const inl_csr *A);
  * same inl_csr. */
 inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y,
                     inl_plan plan);
+
+/* SpMV with a replicated result (the form an iterated SpMV needs): every rank
+ * computes y for its row block (same kernels as inl_spmv) and the blocks are allgathered, so
+ * y_global [n_global] = A * x on every rank.  A must be this rank's block of
+ * inl_partition_rows (the whole CSR without a communicator).  Asynchronous on the ctx stream
+ * for device pointers. */
+inl_status inl_spmv_allgather(inl_ctx ctx, const inl_csr *A, const float *val, const float *x,
+                              float *y_global, inl_plan plan);
 
 /* PageRank (P5@9262, P5@9781; reading R1): A_in = in-edge CSR (rows =
  * destinations, cols = sources), out_degree [n_global].  PR^0 = 1/n;

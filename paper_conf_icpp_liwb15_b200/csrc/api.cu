@@ -4,6 +4,7 @@
 // frontier.cu.  There is no CPU fallback.
 #include <cstdarg>
 #include <cstdio>
+#include <algorithm>
 #include <cstring>
 #include <new>
 
@@ -227,6 +228,20 @@ inl_plan get_plan(inl_ctx ctx, const inl_csr &A, inl_plan user) {
   return p;
 }
 
+// SpMV on a device CSR: the T1 baseline, one of the paper's templates, or the default
+// fused gather (transient plan when plan == NULL).
+void spmv_dispatch(inl_ctx ctx, const inl_csr &d, const float *dval, const float *dx, float *ydev, inl_plan plan) {
+  if (plan && (plan->bins.flags & INL_BINS_THREAD_ONLY)) {
+    INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
+    spmv_thread_only(ctx, d, dval, dx, ydev);
+  } else if (plan && (plan->bins.flags & kTemplateFlags)) {
+    INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
+    spmv_template(ctx, d, plan->bins, dval, dx, ydev);
+  } else {
+    spmv_run(ctx, get_plan(ctx, d, plan), dval, dx, ydev);
+  }
+}
+
 inl_status fail(inl_ctx ctx, inl_status code, const std::string &msg) {
   if (ctx) ctx->last_error = msg;
   g_error = msg;
@@ -239,10 +254,13 @@ inl_status guarded(inl_ctx ctx, F &&f) {
     f();
     return INL_OK;
   } catch (const Error &e) {
+    loop_abort(ctx);  // a failing loopback rank releases its peers (they fail, not hang)
     return fail(ctx, e.code, e.msg);
   } catch (const std::bad_alloc &) {
+    loop_abort(ctx);
     return fail(ctx, INL_ERR_OUT_OF_MEMORY, "host allocation failed");
   } catch (...) {
+    loop_abort(ctx);
     return fail(ctx, INL_ERR_INTERNAL, "unexpected C++ exception");
   }
 }
@@ -284,6 +302,7 @@ void csr_validate(inl_ctx ctx, const inl_csr &A) {
 
 void comm_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
                     const double *d_send, double *d_recv) {
+  if (ctx->loop) return loop_allgather(ctx, send, recv, count, dt, d_send, d_recv);
   INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
   INL_NCCL(ncclGroupStart());
   INL_NCCL(ncclAllGather(send, recv, (size_t)count, dt, ctx->comm, ctx->stream));
@@ -292,6 +311,7 @@ void comm_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, nc
 }
 
 void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op) {
+  if (ctx->loop) return loop_allreduce(ctx, buf, count, dt, op);
   INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
   INL_NCCL(ncclAllReduce(buf, buf, (size_t)count, dt, op, ctx->comm, ctx->stream));
 }
@@ -355,6 +375,7 @@ static void free_ctx(inl_ctx ctx) {
   cudaSetDevice(ctx->device);
   cudaStreamSynchronize(ctx->stream);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
+  if (ctx->loop) loop_release(ctx->loop);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
   delete ctx->tplan;
   delete ctx;  // DevBuf destructors free device scratch
@@ -421,13 +442,23 @@ inl_status inl_comm_init(inl_ctx ctx, const uint8_t uid[128], int32_t nranks, in
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     INL_CHECK(uid != nullptr && nranks >= 1 && rank >= 0 && rank < nranks, "comm_init: bad argument");
-    INL_CHECK(ctx->comm == nullptr, "comm already initialised on this ctx");
+    INL_CHECK(ctx->comm == nullptr && ctx->loop == nullptr, "comm already initialised on this ctx");
     DeviceGuard g(ctx->device);
     ncclUniqueId id;
     memcpy(&id, uid, 128);
     INL_NCCL(ncclCommInitRank(&ctx->comm, nranks, id, rank));
     ctx->nranks = nranks;
     ctx->rank = rank;
+  });
+}
+
+inl_status inl_comm_init_loopback(inl_ctx ctx, inl_loop group, int32_t rank) {
+  if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
+  return guarded(ctx, [&] {
+    INL_CHECK(group != nullptr, "loopback group is NULL");
+    INL_CHECK(ctx->comm == nullptr && ctx->loop == nullptr, "comm already initialised on this ctx");
+    DeviceGuard g(ctx->device);
+    loop_join(ctx, reinterpret_cast<LoopGroup *>(group), rank);
   });
 }
 
@@ -503,15 +534,35 @@ inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float
     const float *dval = stage_in(ctx, ctx->h_val, val, A->nnz);
     const float *dx = stage_in(ctx, ctx->h_x, x, A->n_global);
     StagedOut<float> yo = stage_out(ctx->h_y, y, A->n_rows);
-    if (plan && (plan->bins.flags & INL_BINS_THREAD_ONLY)) {
-      INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
-      spmv_thread_only(ctx, d, dval, dx, yo.dev);
-    } else if (plan && (plan->bins.flags & kTemplateFlags)) {
-      INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
-      spmv_template(ctx, d, plan->bins, dval, dx, yo.dev);
-    } else {
-      spmv_run(ctx, get_plan(ctx, d, plan), dval, dx, yo.dev);
-    }
+    spmv_dispatch(ctx, d, dval, dx, yo.dev, plan);
+    finish_out(ctx, yo);
+  });
+}
+
+inl_status inl_spmv_allgather(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y_global,
+                              inl_plan plan) {
+  if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
+  return guarded(ctx, [&] {
+    check_csr(A);
+    INL_CHECK(A->nnz == 0 || val != nullptr, "val is NULL");
+    INL_CHECK(A->n_global == 0 || (x != nullptr && y_global != nullptr), "x / y_global is NULL");
+    const int64_t n = A->n_global;
+    const int P = has_comm(ctx) ? ctx->nranks : 1;
+    const int64_t B = (n + P - 1) / P;
+    INL_CHECK(has_comm(ctx) || (A->row_begin == 0 && A->n_rows == n), "a partial CSR (row block) needs a communicator");
+    INL_CHECK(A->row_begin == (int64_t)ctx->rank * B && A->n_rows == std::min(B, n - A->row_begin),
+              "row block does not match inl_partition_rows for this rank");
+    DeviceGuard g(ctx->device);
+    inl_csr d = device_csr(ctx, A);
+    const float *dval = stage_in(ctx, ctx->h_val, val, A->nnz);
+    const float *dx = stage_in(ctx, ctx->h_x, x, n);
+    StagedOut<float> yo = stage_out(ctx->h_y, y_global, n);
+    // NCCL's allgather moves equal counts: in place when P divides n, else through a padded copy
+    float *full = B * P == n ? yo.dev : (float *)ctx->s_pad.get(sizeof(float) * (size_t)(B * P));
+    spmv_dispatch(ctx, d, dval, dx, full + A->row_begin, plan);
+    if (has_comm(ctx)) comm_allgather(ctx, full + A->row_begin, full, B, ncclFloat32, nullptr, nullptr);
+    if (full != yo.dev && n > 0)
+      INL_CUDA(cudaMemcpyAsync(yo.dev, full, sizeof(float) * (size_t)n, cudaMemcpyDeviceToDevice, ctx->stream));
     finish_out(ctx, yo);
   });
 }
@@ -524,9 +575,9 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
     INL_CHECK(damping >= 0.0f && damping < 1.0f, "damping must be in [0, 1)");
     INL_CHECK(iterations >= 0, "iterations must be >= 0");
     INL_CHECK(A_in->n_global == 0 || (out_degree && rank), "out_degree/rank is NULL");
-    INL_CHECK(ctx->comm != nullptr || (A_in->row_begin == 0 && A_in->n_rows == A_in->n_global),
+    INL_CHECK(has_comm(ctx) || (A_in->row_begin == 0 && A_in->n_rows == A_in->n_global),
               "a partial CSR (row block) needs inl_comm_init");
-    INL_CHECK(ctx->comm == nullptr || ctx->nranks == 1 ||
+    INL_CHECK(!has_comm(ctx) || ctx->nranks == 1 ||
                   A_in->row_begin == (int64_t)ctx->rank * ((A_in->n_global + ctx->nranks - 1) / ctx->nranks),
               "row block does not match inl_partition_rows for this rank");
     DeviceGuard g(ctx->device);
@@ -550,7 +601,7 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
     INL_CHECK(source >= 0 && source < G->n_global, "source out of range");
     INL_CHECK(G->nnz == 0 || w != nullptr, "w is NULL");
     INL_CHECK(dist != nullptr, "dist is NULL");
-    INL_CHECK(ctx->comm != nullptr || (G->row_begin == 0 && G->n_rows == G->n_global),
+    INL_CHECK(has_comm(ctx) || (G->row_begin == 0 && G->n_rows == G->n_global),
               "a partial CSR (row block) needs inl_comm_init");
     DeviceGuard g(ctx->device);
     inl_csr d = device_csr(ctx, G);
@@ -571,7 +622,7 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
     check_csr(G);
     INL_CHECK(source >= 0 && source < G->n_global, "source out of range");
     INL_CHECK(level != nullptr, "level is NULL");
-    INL_CHECK(ctx->comm != nullptr || (G->row_begin == 0 && G->n_rows == G->n_global),
+    INL_CHECK(has_comm(ctx) || (G->row_begin == 0 && G->n_rows == G->n_global),
               "a partial CSR (row block) needs inl_comm_init");
     DeviceGuard g(ctx->device);
     inl_csr d = device_csr(ctx, G);

@@ -1,11 +1,23 @@
-// comm.h — NCCL exchange used by the multi-GPU row-block path.
+// comm.h — the per-iteration exchange of the multi-GPU row-block path (SURVEY §8a row
+// a12): NCCL over NVLink between processes, or the loopback group (loopback.cu) between
+// row-block contexts on one device.  Same calls, same semantics.
 #pragma once
 #include "inl_internal.cuh"
 
 namespace inl {
+// true when the ctx is one rank of a row-block job (NCCL comm or loopback group; also P = 1)
+inline bool has_comm(inl_ctx ctx) { return ctx->comm != nullptr || ctx->loop != nullptr; }
 // In-place-capable allgather of `count` elements per rank (recv holds nranks*count),
 // optionally grouped with an allgather of one double per rank (d_send -> d_recv).
 void comm_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
                     const double *d_send, double *d_recv);
+// In-place allreduce.
 void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op);
+// loopback.cu
+void loop_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
+                    const double *d_send, double *d_recv);
+void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op);
+void loop_join(inl_ctx ctx, LoopGroup *g, int rank);
+void loop_release(LoopGroup *g);
+void loop_abort(inl_ctx ctx);
 }  // namespace inl

@@ -901,7 +901,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
               uint32_t *dist, inl_stats *stats) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
-  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
   // the device-driven loop (sssp_run_dyn) is opt-in: measured 8.5 ms vs 8.0 ms per scale-23
   // source for the host-driven one (profiles/r01/sssp_devloop.txt) — its 4 launches per
   // step cost more than the ~40 host round trips they save
@@ -1009,7 +1009,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
              inl_stats *stats, bool symmetric) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
-  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
   uint32_t *bm = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * ((n + 31) / 32 + 1));

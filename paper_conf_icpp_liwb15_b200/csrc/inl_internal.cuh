@@ -106,6 +106,7 @@ struct CbPlan {
 }  // namespace inl
 
 namespace inl {
+struct LoopGroup;  // loopback.cu: P row-block contexts on one device standing in for NCCL
 // Per-kernel launch timer (inl_ktimer_*): event pairs pending on the ctx stream, resolved
 // into (launches, ms) totals when read.
 struct KTimer {
@@ -132,10 +133,13 @@ struct inl_ctx_s {
   int num_sms = 148;
   std::string last_error;
   ncclComm_t comm = nullptr;
+  inl::LoopGroup *loop = nullptr;  // loopback group (inl_comm_init_loopback) instead of NCCL
   int nranks = 1, rank = 0;
   // scratch
   inl::DevBuf s_tmp, s_a, s_b, s_c, s_d, s_e, s_f, s_g;
   inl::DevBuf h_rp, h_ci, h_val, h_x, h_y, h_w, h_od;  // host-staging device copies
+  inl::DevBuf s_loop;                                  // loopback allreduce scratch
+  inl::DevBuf s_pad;                                   // padded replicated vectors (P > 1)
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)

@@ -232,7 +232,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
     return;
   }
   const int P = ctx->nranks;
-  const bool DIST = ctx->comm != nullptr;  // row-block mode with NCCL exchange (also P = 1)
+  const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
   const int64_t B = DIST ? (n + P - 1) / P : n;  // row block (inl_partition_rows)
   const int64_t npad = B * P;
   pr_compact(ctx, p, out_degree, B, DIST ? P : 1);

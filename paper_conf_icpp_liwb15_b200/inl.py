@@ -84,6 +84,10 @@ def lib() -> C.CDLL:
         L.inl_partition_rows.argtypes = [i64, i32, vp]
         L.inl_nccl_unique_id.argtypes = [vp]
         L.inl_comm_init.argtypes = [vp, vp, i32, i32]
+        L.inl_loop_create.argtypes = [i32, C.POINTER(vp)]
+        L.inl_loop_destroy.argtypes = [vp]
+        L.inl_comm_init_loopback.argtypes = [vp, vp, i32]
+        L.inl_spmv_allgather.argtypes = [vp, C.POINTER(CsrT), vp, vp, vp, vp]
         L.inl_plan_create.argtypes = [vp, C.POINTER(CsrT), C.POINTER(BinsT), C.POINTER(vp)]
         L.inl_plan_get_info.argtypes = [vp, C.POINTER(PlanInfoT)]
         L.inl_plan_destroy.argtypes = [vp]
@@ -96,7 +100,8 @@ def lib() -> C.CDLL:
         L.inl_ktimer_enable.argtypes = [vp, i32]
         L.inl_ktimer_read.argtypes = [vp, C.c_char_p, C.POINTER(i64), C.POINTER(C.c_double)]
         for f in ("inl_ctx_create", "inl_ctx_set_stream", "inl_ctx_destroy", "inl_partition_rows",
-                  "inl_nccl_unique_id", "inl_comm_init", "inl_plan_create", "inl_plan_get_info",
+                  "inl_nccl_unique_id", "inl_comm_init", "inl_loop_create", "inl_loop_destroy",
+                  "inl_comm_init_loopback", "inl_spmv_allgather", "inl_plan_create", "inl_plan_get_info",
                   "inl_plan_destroy", "inl_csr_validate", "inl_spmv", "inl_pagerank", "inl_sssp", "inl_bfs",
                   "inl_ktimer_enable", "inl_ktimer_read"):
             getattr(L, f).restype = C.c_int
@@ -179,6 +184,11 @@ class Ctx:
         _check(lib().inl_comm_init(self.handle, uid.ctypes.data, nranks, rank), self)
         self.nranks, self.rank = nranks, rank
 
+    def comm_init_loopback(self, group: "LoopGroup", rank: int) -> None:
+        """Join a loopback group as `rank` (row-block contexts on one device)."""
+        _check(lib().inl_comm_init_loopback(self.handle, group.handle, int(rank)), self)
+        self.nranks, self.rank = group.nranks, int(rank)
+
     def ktimer_enable(self, on: bool = True) -> None:
         """Bracket the main kernels' launches with CUDA events (measurement only)."""
         _check(lib().inl_ktimer_enable(self.handle, 1 if on else 0), self)
@@ -192,6 +202,29 @@ class Ctx:
     def close(self) -> None:
         if getattr(self, "handle", None):
             lib().inl_ctx_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class LoopGroup:
+    """Host object of a loopback communicator for `nranks` contexts on one device
+    (inl_loop_create).  Drive each member ctx from its own thread."""
+
+    def __init__(self, nranks: int):
+        h = C.c_void_p()
+        rc = lib().inl_loop_create(int(nranks), C.byref(h))
+        if rc != INL_OK:
+            raise InlError(rc, "inl_loop_create")
+        self.handle, self.nranks = h, int(nranks)
+
+    def close(self) -> None:
+        if getattr(self, "handle", None):
+            lib().inl_loop_destroy(self.handle)
             self.handle = None
 
     def __del__(self):
@@ -273,6 +306,16 @@ def spmv(ctx: Ctx, A: Csr, val, x, y, plan: Plan | None = None):
     s = A.struct()
     _check(lib().inl_spmv(ctx.handle, C.byref(s), _ptr(val), _ptr(x), _ptr(y), _plan_handle(plan)), ctx)
     return y
+
+
+def spmv_allgather(ctx: Ctx, A: Csr, val, x, y_global, plan: Plan | None = None):
+    """y_global[n_global] = A * x replicated on every rank: this rank's row block, then the
+    allgather of the blocks."""
+    ctx.sync_stream()
+    s = A.struct()
+    _check(lib().inl_spmv_allgather(ctx.handle, C.byref(s), _ptr(val), _ptr(x), _ptr(y_global),
+                                    _plan_handle(plan)), ctx)
+    return y_global
 
 
 def pagerank(ctx: Ctx, A_in: Csr, out_degree, rank, damping: float = 0.85, iterations: int = 20,

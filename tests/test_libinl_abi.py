@@ -82,3 +82,19 @@ def test_ctx_create_without_gpu_reports_cuda_error():
     h = C.c_void_p()
     assert inl.lib().inl_ctx_create(C.byref(h), 0, None) == 3  # INL_ERR_CUDA
     assert "cuda" in inl.lib().inl_last_error(None).decode().lower()
+
+
+def test_loop_group_host_object():
+    """The loopback communicator's host object needs no GPU: create / destroy / bad sizes."""
+    L = inl.lib()
+    for p in (1, 2, 8, 64):
+        g = inl.LoopGroup(p)
+        assert g.nranks == p
+        g.close()
+    h = C.c_void_p()
+    assert L.inl_loop_create(0, C.byref(h)) == 1
+    assert L.inl_loop_create(65, C.byref(h)) == 1
+    assert L.inl_loop_destroy(None) == 0
+    s = inl.CsrT(0, 0, 0, 0, None, None)
+    assert L.inl_spmv_allgather(None, C.byref(s), None, None, None, None) == 1
+    assert L.inl_comm_init_loopback(None, None, 0) == 1
