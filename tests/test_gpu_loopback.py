@@ -127,7 +127,7 @@ def test_spmv_integer_bit_exact(g12_dir, P, use_plan):
 
 @pytest.mark.parametrize("P", PS)
 def test_spmv_float_within_1e5(P):
-    g = inlgen.host_build(16, 16, seed=inlgen.SEED_GRAPH)
+    g = inlgen.host_build(18, 16, seed=inlgen.SEED_GRAPH)
     val = inlgen.values_host(g.row_ptr, g.col_idx)
     x = inlgen.vector_host(g.n_global)
     ref = oracle.spmv(g.row_ptr, g.col_idx, val, x)
