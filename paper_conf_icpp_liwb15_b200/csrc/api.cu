@@ -301,19 +301,32 @@ void csr_validate(inl_ctx ctx, const inl_csr &A) {
 }
 
 void comm_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
-                    const double *d_send, double *d_recv) {
-  if (ctx->loop) return loop_allgather(ctx, send, recv, count, dt, d_send, d_recv);
+                    const double *d_send, double *d_recv, cudaStream_t st) {
+  if (!st) st = ctx->stream;
+  if (ctx->loop) return loop_allgather(ctx, send, recv, count, dt, d_send, d_recv, st);
   INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
   INL_NCCL(ncclGroupStart());
-  INL_NCCL(ncclAllGather(send, recv, (size_t)count, dt, ctx->comm, ctx->stream));
-  if (d_send) INL_NCCL(ncclAllGather(d_send, d_recv, 1, ncclFloat64, ctx->comm, ctx->stream));
+  INL_NCCL(ncclAllGather(send, recv, (size_t)count, dt, ctx->comm, st));
+  if (d_send) INL_NCCL(ncclAllGather(d_send, d_recv, 1, ncclFloat64, ctx->comm, st));
   INL_NCCL(ncclGroupEnd());
 }
 
-void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op) {
-  if (ctx->loop) return loop_allreduce(ctx, buf, count, dt, op);
+void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op, cudaStream_t st) {
+  if (!st) st = ctx->stream;
+  if (ctx->loop) return loop_allreduce(ctx, buf, count, dt, op, st);
   INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
-  INL_NCCL(ncclAllReduce(buf, buf, (size_t)count, dt, op, ctx->comm, ctx->stream));
+  INL_NCCL(ncclAllReduce(buf, buf, (size_t)count, dt, op, ctx->comm, st));
+}
+
+cudaStream_t comm_stream(inl_ctx ctx) {
+  if (!ctx->comm_stream) INL_CUDA(cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking));
+  return ctx->comm_stream;
+}
+
+cudaEvent_t ctx_event(inl_ctx ctx, int i) {
+  INL_CHECK(i >= 0 && i < kCtxEvents, "ctx_event: index out of range");
+  if (!ctx->events[i]) INL_CUDA(cudaEventCreateWithFlags(&ctx->events[i], cudaEventDisableTiming));
+  return ctx->events[i];
 }
 
 }  // namespace inl
@@ -376,6 +389,12 @@ static void free_ctx(inl_ctx ctx) {
   cudaStreamSynchronize(ctx->stream);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   if (ctx->loop) loop_release(ctx->loop);
+  if (ctx->comm_stream) {
+    cudaStreamSynchronize(ctx->comm_stream);
+    cudaStreamDestroy(ctx->comm_stream);
+  }
+  for (cudaEvent_t e : ctx->events)
+    if (e) cudaEventDestroy(e);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
   delete ctx->tplan;
   delete ctx;  // DevBuf destructors free device scratch

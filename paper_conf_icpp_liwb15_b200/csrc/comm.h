@@ -9,14 +9,19 @@ namespace inl {
 inline bool has_comm(inl_ctx ctx) { return ctx->comm != nullptr || ctx->loop != nullptr; }
 // In-place-capable allgather of `count` elements per rank (recv holds nranks*count),
 // optionally grouped with an allgather of one double per rank (d_send -> d_recv).
+// st: the stream the exchange is ordered on (nullptr = the ctx stream).
 void comm_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
-                    const double *d_send, double *d_recv);
+                    const double *d_send, double *d_recv, cudaStream_t st = nullptr);
 // In-place allreduce.
-void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op);
+void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op,
+                    cudaStream_t st = nullptr);
+// the ctx's second stream (created on first use): exchanges overlapped with the gather
+cudaStream_t comm_stream(inl_ctx ctx);
+cudaEvent_t ctx_event(inl_ctx ctx, int i);  // ctx-owned timing-free events, i < kCtxEvents
 // loopback.cu
 void loop_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
-                    const double *d_send, double *d_recv);
-void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op);
+                    const double *d_send, double *d_recv, cudaStream_t st);
+void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op, cudaStream_t st);
 void loop_join(inl_ctx ctx, LoopGroup *g, int rank);
 void loop_release(LoopGroup *g);
 void loop_abort(inl_ctx ctx);

@@ -448,7 +448,7 @@ __global__ void __launch_bounds__(256) k_gather_thread_only(int64_t n_rows, Gath
 void build_xhot(inl_ctx ctx, inl_plan p, const float *x, const int32_t *hot_cols = nullptr, int64_t n_hot = -1);
 
 template <int E, bool VALS, class Epi, int NWARP = 256 / E>
-void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
+void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi, int max_ctas = 0) {
   const size_t smem = (size_t)gp.n_hot * 4 + 16;  // xs[0] is read (then discarded) by cold gathers
   auto kern = k_gather<E, VALS, Epi, NWARP>;
   static size_t configured[kMaxDevices] = {};  // per instantiation AND device (the attribute is per device)
@@ -457,7 +457,7 @@ void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, con
     INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     cf = smem;
   }
-  int64_t grid = ctx->num_sms;
+  int64_t grid = max_ctas > 0 && max_ctas < ctx->num_sms ? max_ctas : ctx->num_sms;
   const int64_t need = (gp.n_items + NWARP - 1) / NWARP;
   if (grid > need) grid = need;
   KScope ks(ctx, "k_gather");
@@ -474,6 +474,16 @@ inline int gather_entries_per_lane() {
   return e;
 }
 
+// A sub-range of a plan's work items for one launch (PageRank's pipelined sub-blocks): items
+// [items, items + n) write their dangling partials to dpart[0, n); max_ctas caps the grid
+// (leaves SMs to a concurrent NCCL kernel); skip_xhot: x_hot is already current.
+struct GatherRange {
+  const WorkItem *items = nullptr;  // nullptr: every item of the plan
+  int64_t n = 0;
+  int max_ctas = 0;
+  bool skip_xhot = false;
+};
+
 // Host-side launcher for one full gather (tiles + long-row chunks) on a plan; x is the
 // dense vector (n_global) whose hot part is copied to the plan's x_hot first.
 // col_over / hot_over: a column space other than the plan's (PageRank's compacted one).
@@ -482,17 +492,18 @@ inline int gather_entries_per_lane() {
 template <bool VALS, class Epi>
 void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &epi, double *dpart,
                    const int32_t *col_over = nullptr, const int32_t *hot_over = nullptr,
-                   const CbPlan *cb = nullptr, int64_t n_hot_over = -1) {
+                   const CbPlan *cb = nullptr, int64_t n_hot_over = -1, const GatherRange *range = nullptr) {
   if (p->n_items == 0) return;
   const int64_t n_hot = n_hot_over >= 0 ? n_hot_over : p->n_hot;
   const bool use_cb = cb && cb->active;
-  const int64_t n_items = use_cb ? cb->n_items : p->n_items;
+  const bool ranged = range && range->items;
+  const int64_t n_items = ranged ? range->n : use_cb ? cb->n_items : p->n_items;
   GatherArgs a = a_in;
   if (col_over) a.col_idx = col_over;
   else if (p->n_hot > 0) a.col_idx = (const int32_t *)p->pcol.p;  // hot columns remapped
   if (n_items > 0) {
     GatherPlan gp;
-    gp.items = (const WorkItem *)(use_cb ? cb->items.p : p->items.p);
+    gp.items = ranged ? range->items : (const WorkItem *)(use_cb ? cb->items.p : p->items.p);
     gp.n_items = (int)n_items;
     gp.partials = (float *)p->partials.p;
     gp.tickets = (int *)p->tickets.p;
@@ -505,16 +516,17 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     // each launch advances the counter by exactly n_items (successful grabs + one failing
     // grab per active warp), so the next launch's base is known on the host: no reset
     gp.base = p->ticket_base;
-    build_xhot(ctx, p, a.x, hot_over, n_hot);
+    if (!(ranged && range->skip_xhot)) build_xhot(ctx, p, a.x, hot_over, n_hot);
     a.vec = ((uintptr_t)a.col_idx % 32 == 0) && (!VALS || (uintptr_t)a.val % 32 == 0);
     static int w24 = -1;
     if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;
-    if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi);
-    else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi);
-    else launch_gather_t<8, VALS>(ctx, gp, a, epi);
+    const int mc = ranged ? range->max_ctas : 0;
+    if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi, mc);
+    else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi, mc);
+    else launch_gather_t<8, VALS>(ctx, gp, a, epi, mc);
     p->ticket_base += (unsigned long long)n_items;  // only once the launch was accepted
   }
-  if (use_cb) launch_cb<VALS>(ctx, *cb, a_in.val, a_in.x, epi, dpart ? dpart + n_items : nullptr);
+  if (use_cb && !ranged) launch_cb<VALS>(ctx, *cb, a_in.val, a_in.x, epi, dpart ? dpart + n_items : nullptr);
 }
 
 // number of dangling partials launch_gather writes

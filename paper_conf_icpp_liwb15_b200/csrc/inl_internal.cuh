@@ -13,6 +13,7 @@ namespace inl {
 
 constexpr int kTileRows = 256;  // max rows per SpMV/PR warp tile
 constexpr int kMaxDevices = 64;  // per-device caches of kernel attributes
+constexpr int kCtxEvents = 16;   // events a ctx keeps for cross-stream ordering
 
 // One unit of work of the fused gather kernel (one warp): a tile (j < 0: rows [r0, r1),
 // all of degree <= t_warp, nonzeros [s, e), tile index t into the plan's non-empty-row
@@ -134,6 +135,8 @@ struct inl_ctx_s {
   std::string last_error;
   ncclComm_t comm = nullptr;
   inl::LoopGroup *loop = nullptr;  // loopback group (inl_comm_init_loopback) instead of NCCL
+  cudaStream_t comm_stream = nullptr;  // second stream: exchanges overlapped with the gather
+  cudaEvent_t events[inl::kCtxEvents] = {};
   int nranks = 1, rank = 0;
   // scratch
   inl::DevBuf s_tmp, s_a, s_b, s_c, s_d, s_e, s_f, s_g;
@@ -182,7 +185,11 @@ struct inl_plan_s {
   // PageRank: contributions live in the compacted space of non-dangling vertices
   // (every column of an in-CSR is a page with out-links), cached per out_degree array
   const int32_t *pr_od = nullptr;
-  int64_t pr_bc = 0;           // compact slots per rank block
+  int64_t pr_bc = 0;           // compact slots per (rank block, sub-block) group
+  int pr_P = 0, pr_K = 0;      // ranks and row sub-blocks the compaction was built for
+  int64_t pr_Bs = 0;           // sub-block width in rows (a multiple of kTileRows)
+  std::vector<int64_t> pr_iofs;  // [pr_K + 1] first work item of each sub-block in pr_items
+  inl::DevBuf pr_items;        // WorkItem [n_items] grouped by sub-block (pr_K > 1)
   inl::DevBuf pr_cidx;         // int32 [n_global]: exchange-space index, -1 if dangling
   inl::DevBuf pr_col;          // int32 [nnz]: gather columns in the compact space (hot kept)
   inl::DevBuf pr_hot;          // int32 [pr_nhot]: hot slots in the compact space

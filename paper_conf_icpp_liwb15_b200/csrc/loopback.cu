@@ -111,84 +111,79 @@ size_t dt_size(ncclDataType_t dt) {
 }
 
 template <class T>
-void launch_reduce(inl_ctx ctx, LoopGroup *g, ncclRedOp_t op, int64_t count, void *out) {
+void launch_reduce(inl_ctx ctx, LoopGroup *g, ncclRedOp_t op, int64_t count, void *out, cudaStream_t st) {
   PeerPtrs<T> pp{};
   for (int q = 0; q < g->nranks; ++q) pp.p[q] = (const T *)g->src[q];
   int64_t grid = (count + 255) / 256;
   if (grid > (int64_t)ctx->num_sms * 8) grid = (int64_t)ctx->num_sms * 8;
   if (grid < 1) grid = 1;
   T *o = (T *)out;
-  if (op == ncclMin) k_loop_reduce<T, 0><<<(int)grid, 256, 0, ctx->stream>>>(pp, g->nranks, count, o);
-  else if (op == ncclMax) k_loop_reduce<T, 1><<<(int)grid, 256, 0, ctx->stream>>>(pp, g->nranks, count, o);
-  else if (op == ncclSum) k_loop_reduce<T, 2><<<(int)grid, 256, 0, ctx->stream>>>(pp, g->nranks, count, o);
+  if (op == ncclMin) k_loop_reduce<T, 0><<<(int)grid, 256, 0, st>>>(pp, g->nranks, count, o);
+  else if (op == ncclMax) k_loop_reduce<T, 1><<<(int)grid, 256, 0, st>>>(pp, g->nranks, count, o);
+  else if (op == ncclSum) k_loop_reduce<T, 2><<<(int)grid, 256, 0, st>>>(pp, g->nranks, count, o);
   else raise(INL_ERR_UNSUPPORTED, "loopback: unsupported reduction op");
   INL_CUDA(cudaGetLastError());
 }
 
 // phase 1: publish + ready event + barrier + wait for the peers' inputs
-void phase_in(inl_ctx ctx, LoopGroup *g, const void *src, void *dst, const double *dsrc) {
+void phase_in(inl_ctx ctx, LoopGroup *g, const void *src, void *dst, const double *dsrc, cudaStream_t st) {
   const int r = ctx->rank;
   g->src[r] = src;
   g->dst[r] = dst;
   g->dsrc[r] = dsrc;
-  INL_CUDA(cudaEventRecord(g->ready[r], ctx->stream));
+  INL_CUDA(cudaEventRecord(g->ready[r], st));
   g->barrier();
   for (int q = 0; q < g->nranks; ++q)
-    if (q != r) INL_CUDA(cudaStreamWaitEvent(ctx->stream, g->ready[q], 0));
+    if (q != r) INL_CUDA(cudaStreamWaitEvent(st, g->ready[q], 0));
 }
 
 // phase 2: done event + barrier + wait until no peer still reads this rank's buffers
-void phase_out(inl_ctx ctx, LoopGroup *g) {
+void phase_out(inl_ctx ctx, LoopGroup *g, cudaStream_t st) {
   const int r = ctx->rank;
-  INL_CUDA(cudaEventRecord(g->done[r], ctx->stream));
+  INL_CUDA(cudaEventRecord(g->done[r], st));
   g->barrier();
   for (int q = 0; q < g->nranks; ++q)
-    if (q != r) INL_CUDA(cudaStreamWaitEvent(ctx->stream, g->done[q], 0));
+    if (q != r) INL_CUDA(cudaStreamWaitEvent(st, g->done[q], 0));
 }
 
 }  // namespace
 
 void loop_allgather(inl_ctx ctx, const void *send, void *recv, int64_t count, ncclDataType_t dt,
-                    const double *d_send, double *d_recv) {
+                    const double *d_send, double *d_recv, cudaStream_t st) {
   LoopGroup *g = ctx->loop;
   const int r = ctx->rank, P = g->nranks;
   const size_t bytes = dt_size(dt) * (size_t)count;
-  phase_in(ctx, g, send, recv, d_send);
+  phase_in(ctx, g, send, recv, d_send, st);
   for (int q = 0; q < P; ++q) {
     char *to = (char *)recv + (size_t)q * bytes;
     if (bytes && to != g->src[q])  // in place for q == r: nothing to copy
-      INL_CUDA(cudaMemcpyAsync(to, g->src[q], bytes, cudaMemcpyDeviceToDevice, ctx->stream));
-    if (d_send) INL_CUDA(cudaMemcpyAsync(d_recv + q, g->dsrc[q], sizeof(double), cudaMemcpyDeviceToDevice, ctx->stream));
+      INL_CUDA(cudaMemcpyAsync(to, g->src[q], bytes, cudaMemcpyDeviceToDevice, st));
+    if (d_send) INL_CUDA(cudaMemcpyAsync(d_recv + q, g->dsrc[q], sizeof(double), cudaMemcpyDeviceToDevice, st));
   }
   (void)r;
-  phase_out(ctx, g);
+  phase_out(ctx, g, st);
 }
 
-void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op) {
+void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, ncclRedOp_t op, cudaStream_t st) {
   LoopGroup *g = ctx->loop;
   const size_t es = dt_size(dt);
   void *tmp = ctx->s_loop.get(es * (size_t)(count > 0 ? count : 1));
-  phase_in(ctx, g, buf, buf, nullptr);
+  phase_in(ctx, g, buf, buf, nullptr, st);
   if (count > 0) {
     switch (dt) {
-      case ncclUint8: launch_reduce<uint8_t>(ctx, g, op, count, tmp); break;
-      case ncclInt8: launch_reduce<int8_t>(ctx, g, op, count, tmp); break;
-      case ncclUint32: launch_reduce<uint32_t>(ctx, g, op, count, tmp); break;
-      case ncclInt32: launch_reduce<int32_t>(ctx, g, op, count, tmp); break;
-      case ncclUint64: launch_reduce<unsigned long long>(ctx, g, op, count, tmp); break;
-      case ncclInt64: launch_reduce<long long>(ctx, g, op, count, tmp); break;
-      case ncclFloat32: launch_reduce<float>(ctx, g, op, count, tmp); break;
-      case ncclFloat64: launch_reduce<double>(ctx, g, op, count, tmp); break;
+      case ncclUint8: launch_reduce<uint8_t>(ctx, g, op, count, tmp, st); break;
+      case ncclInt8: launch_reduce<int8_t>(ctx, g, op, count, tmp, st); break;
+      case ncclUint32: launch_reduce<uint32_t>(ctx, g, op, count, tmp, st); break;
+      case ncclInt32: launch_reduce<int32_t>(ctx, g, op, count, tmp, st); break;
+      case ncclUint64: launch_reduce<unsigned long long>(ctx, g, op, count, tmp, st); break;
+      case ncclInt64: launch_reduce<long long>(ctx, g, op, count, tmp, st); break;
+      case ncclFloat32: launch_reduce<float>(ctx, g, op, count, tmp, st); break;
+      case ncclFloat64: launch_reduce<double>(ctx, g, op, count, tmp, st); break;
       default: raise(INL_ERR_UNSUPPORTED, "loopback: unsupported datatype for allreduce");
     }
   }
-  phase_out(ctx, g);  // every peer has read this rank's buf: overwrite it in place
-  if (count > 0) INL_CUDA(cudaMemcpyAsync(buf, tmp, es * (size_t)count, cudaMemcpyDeviceToDevice, ctx->stream));
-}
-
-void loop_barrier(inl_ctx ctx) {
-  phase_in(ctx, ctx->loop, nullptr, nullptr, nullptr);
-  phase_out(ctx, ctx->loop);
+  phase_out(ctx, g, st);  // every peer has read this rank's buf: overwrite it in place
+  if (count > 0) INL_CUDA(cudaMemcpyAsync(buf, tmp, es * (size_t)count, cudaMemcpyDeviceToDevice, st));
 }
 
 void loop_abort(inl_ctx ctx) {

@@ -76,36 +76,54 @@ __global__ void k_nd_flags(const int32_t *__restrict__ od, int64_t n, int32_t *_
     f[v] = v < n && od[v] > 0;
 }
 
-// exchange-space index: block q = v / B holds slots [q*Bc, (q+1)*Bc); -1 for dangling pages
-__global__ void k_cidx(const int32_t *__restrict__ od, const int32_t *__restrict__ pos, int64_t n, int64_t B,
-                       int64_t Bc, int32_t *__restrict__ cidx) {
+// Exchange-space layout (DESIGN.md §5 "PageRank exchange"): rank block q = v / B is cut into
+// K row sub-blocks of Bs rows; group (q, k) holds its pages with out-links in slots
+//   k * (P * Bck) + q * Bck + i,   i < Bck,
+// so sub-block k of every rank is one contiguous, rank-major range: its allgather is NCCL's
+// in-place layout and can start as soon as sub-block k's gather is done.  K = 1 is the plain
+// rank-major layout q * Bck + i.
+struct GroupMap {
+  int64_t B, Bs, Bck;
+  int P;
+  __device__ __forceinline__ int64_t q_of(int64_t v) const { return v / B; }
+  __device__ __forceinline__ int64_t k_of(int64_t v, int64_t q) const { return (v - q * B) / Bs; }
+  __device__ __forceinline__ int64_t start(int64_t q, int64_t k) const { return q * B + k * Bs; }
+  __device__ __forceinline__ int64_t slot(int64_t q, int64_t k, int64_t i) const {
+    return k * ((int64_t)P * Bck) + q * Bck + i;
+  }
+};
+
+// vertex order inside a group: i = rank among the group's pages with out-links
+__global__ void k_cidx(const int32_t *__restrict__ od, const int32_t *__restrict__ pos, int64_t n, GroupMap gm,
+                       int32_t *__restrict__ cidx) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
        v += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t q = v / B;
-    cidx[v] = od[v] > 0 ? (int32_t)(q * Bc + (pos[v] - pos[q * B])) : -1;
+    const int64_t q = gm.q_of(v), k = gm.k_of(v, q);
+    cidx[v] = od[v] > 0 ? (int32_t)gm.slot(q, k, pos[v] - pos[gm.start(q, k)]) : -1;
   }
 }
 
-// degree order: key = (rank block q, ~out_degree) so that, after a stable sort, block q's
-// pages with out-links come first in descending out-degree (ties by id), dangling last
-__global__ void k_deg_keys(const int32_t *__restrict__ od, int64_t n, int64_t B, uint64_t *__restrict__ key,
-                           int32_t *__restrict__ ids) {
+// degree order: key = (group, ~out_degree) so that, after a stable sort, group g's pages with
+// out-links come first in descending out-degree (ties by id), dangling last
+__global__ void k_deg_keys(const int32_t *__restrict__ od, int64_t n, GroupMap gm, int K,
+                           uint64_t *__restrict__ key, int32_t *__restrict__ ids) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
        v += (int64_t)gridDim.x * blockDim.x) {
-    key[v] = ((uint64_t)(v / B) << 32) | (uint64_t)(~(uint32_t)max(od[v], 0));
+    const int64_t q = gm.q_of(v), g = q * K + gm.k_of(v, q);
+    key[v] = ((uint64_t)g << 32) | (uint64_t)(~(uint32_t)max(od[v], 0));
     ids[v] = (int32_t)v;
   }
 }
 
-// slot of the i-th vertex of the sorted order within its block (blocks are contiguous runs
-// of B positions in the sorted order)
+// slot of the i-th vertex of the sorted order within its group (groups are contiguous runs of
+// vertex ids, so group (q, k) occupies sorted positions [start(q, k), ...))
 __global__ void k_cidx_sorted(const int32_t *__restrict__ od, const int32_t *__restrict__ ids, int64_t n,
-                              int64_t B, int64_t Bc, int32_t *__restrict__ cidx) {
+                              GroupMap gm, int32_t *__restrict__ cidx) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t v = ids[i];
-    const int64_t q = v / B;
-    cidx[v] = od[v] > 0 ? (int32_t)(q * Bc + (i - q * B)) : -1;
+    const int64_t q = gm.q_of(v), k = gm.k_of(v, q);
+    cidx[v] = od[v] > 0 ? (int32_t)gm.slot(q, k, i - gm.start(q, k)) : -1;
   }
 }
 
@@ -144,29 +162,41 @@ int grid_for(int64_t n, int sms) {
 }  // namespace
 
 // Compact (exchange-space) numbering of the pages with out-links, the gather columns in
-// that space, and the slots per rank block.  Cached in the plan per out_degree array.
-// Inside a rank block the slots follow descending out-degree (= how often a page's
-// contribution is gathered), so the frequently read contributions share cache lines
-// and stay L2-resident; INL_PR_ORDER=vertex keeps vertex order (measurement switch).
-static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, int P) {
-  if (p->pr_od == od) return;
+// that space, and the slots per (rank block, sub-block) group.  Cached in the plan per
+// (out_degree array, P, K).  Inside a group the slots follow descending out-degree (= how
+// often a page's contribution is gathered), so the frequently read contributions share cache
+// lines and stay L2-resident; INL_PR_ORDER=vertex keeps vertex order (measurement switch).
+static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, int P, int K) {
+  if (p->pr_od == od && p->pr_P == P && p->pr_K == K) return;
   cudaStream_t st = ctx->stream;
   const int64_t n = p->n_global;
+  // sub-block width: a multiple of kTileRows, so that no row tile of the plan straddles two
+  const int64_t Bs = K > 1 ? ((B + K - 1) / K + kTileRows - 1) / kTileRows * kTileRows : std::max<int64_t>(B, 1);
   int32_t *flags = (int32_t *)ctx->s_e.get(sizeof(int32_t) * (n + 1));
   int32_t *pos = (int32_t *)ctx->s_f.get(sizeof(int32_t) * (n + 1));
   k_nd_flags<<<grid_for(n + 1, ctx->num_sms), 256, 0, st>>>(od, n, flags);
   size_t need = 0;
   INL_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, need, flags, pos, n + 1, st));
   INL_CUDA(cub::DeviceScan::ExclusiveSum(ctx->s_tmp.get(need), need, flags, pos, n + 1, st));
-  std::vector<int32_t> at(P + 1);
-  for (int q = 0; q <= P; ++q) {
-    const int64_t v = std::min<int64_t>((int64_t)q * B, n);
-    INL_CUDA(cudaMemcpyAsync(&at[q], pos + v, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-  }
+  // pages with out-links per group = pos[group end] - pos[group start]
+  std::vector<int64_t> gb;  // group boundaries (vertex ids), 2 per group
+  for (int q = 0; q < P; ++q)
+    for (int k = 0; k < K; ++k) {
+      const int64_t hi_q = std::min<int64_t>((int64_t)(q + 1) * B, n);
+      const int64_t lo = std::min<int64_t>((int64_t)q * B + k * Bs, hi_q);
+      const int64_t hi = std::min<int64_t>((int64_t)q * B + (int64_t)(k + 1) * Bs, hi_q);
+      gb.push_back(lo);
+      gb.push_back(hi);
+    }
+  std::vector<int32_t> at(gb.size());
+  for (size_t i = 0; i < gb.size(); ++i)
+    INL_CUDA(cudaMemcpyAsync(&at[i], pos + gb[i], sizeof(int32_t), cudaMemcpyDeviceToHost, st));
   INL_CUDA(cudaStreamSynchronize(st));
-  int64_t bc = 1;
-  for (int q = 0; q < P; ++q) bc = std::max<int64_t>(bc, (int64_t)at[q + 1] - at[q]);
-  p->pr_bc = bc;
+  int64_t bck = 1;
+  for (size_t i = 0; i < gb.size(); i += 2) bck = std::max<int64_t>(bck, (int64_t)at[i + 1] - at[i]);
+  p->pr_bc = bck;
+  p->pr_Bs = Bs;
+  const GroupMap gm{B, Bs, bck, P};
   int32_t *cidx = (int32_t *)p->pr_cidx.get(sizeof(int32_t) * (n > 0 ? n : 1));
   static int vorder = -1;
   if (vorder < 0) {
@@ -174,22 +204,22 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
     vorder = e && std::string(e) == "vertex";
   }
   if (vorder || n <= 1) {
-    k_cidx<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, pos, n, B, bc, cidx);
+    k_cidx<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, pos, n, gm, cidx);
   } else {
     uint64_t *k0 = (uint64_t *)ctx->s_a.get(sizeof(uint64_t) * n);
     uint64_t *k1 = (uint64_t *)ctx->s_b.get(sizeof(uint64_t) * n);
     int32_t *i0 = flags, *i1 = pos;  // the scan results are no longer needed
-    k_deg_keys<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, n, B, k0, i0);
+    k_deg_keys<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, n, gm, K, k0, i0);
     int end_bit = 32;
-    while (end_bit < 64 && ((uint64_t)(P - 1) >> (end_bit - 32))) ++end_bit;
+    while (end_bit < 64 && ((uint64_t)(P * K - 1) >> (end_bit - 32))) ++end_bit;
     cub::DoubleBuffer<uint64_t> kb(k0, k1);
     cub::DoubleBuffer<int32_t> vb(i0, i1);
     size_t sneed = 0;
     INL_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, sneed, kb, vb, n, 0, end_bit, st));
     INL_CUDA(cub::DeviceRadixSort::SortPairs(ctx->s_tmp.get(sneed), sneed, kb, vb, n, 0, end_bit, st));
-    k_cidx_sorted<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, vb.Current(), n, B, bc, cidx);
+    k_cidx_sorted<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(od, vb.Current(), n, gm, cidx);
   }
-  const int32_t zero_slot = (int32_t)(bc * P);
+  const int32_t zero_slot = (int32_t)(bck * P * K);
   const int32_t *src = p->n_hot > 0 ? (const int32_t *)p->pcol.p : p->col_idx;
   int32_t *pc = (int32_t *)p->pr_col.get(sizeof(int32_t) * (p->nnz > 0 ? p->nnz : 1));
   // PageRank's own hot set: the first pr_nhot slots of the plan's (ranked by frequency);
@@ -216,9 +246,38 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
     if (p->nnz > 0)
       k_remap_cols<<<grid_for(p->nnz, ctx->num_sms), 256, 0, st>>>(p->col_idx, p->nnz, cidx, zero_slot, rc);
     INL_CUDA(cudaGetLastError());
-    cb_build(p, p->pr_cb, rc, bc * P + 1, /*sort_rows=*/!vorder);
+    cb_build(p, p->pr_cb, rc, bck * P * K + 1, /*sort_rows=*/!vorder);
+  }
+  // the gather's work items grouped by sub-block (stable: longest-first inside each), so that
+  // sub-block k is one launch over items [pr_iofs[k], pr_iofs[k+1])
+  p->pr_iofs.assign(K + 1, 0);
+  p->pr_iofs[K] = p->n_items;
+  if (K > 1 && p->n_items > 0) {
+    std::vector<WorkItem> h(p->n_items), o;
+    INL_CUDA(cudaMemcpyAsync(h.data(), p->items.p, sizeof(WorkItem) * h.size(), cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    o.reserve(h.size());
+    for (int k = 0; k < K; ++k) {
+      p->pr_iofs[k] = (int64_t)o.size();
+      for (const WorkItem &w : h)
+        if (std::min<int64_t>(w.r0 / Bs, K - 1) == k) o.push_back(w);
+    }
+    INL_CHECK(o.size() == h.size(), "pagerank: sub-block item split lost items");
+    WorkItem *d = (WorkItem *)p->pr_items.get(sizeof(WorkItem) * o.size());
+    INL_CUDA(cudaMemcpyAsync(d, o.data(), sizeof(WorkItem) * o.size(), cudaMemcpyHostToDevice, st));
+    INL_CUDA(cudaStreamSynchronize(st));
   }
   p->pr_od = od;
+  p->pr_P = P;
+  p->pr_K = K;
+}
+
+// Row sub-blocks per rank for the pipelined exchange (P > 1): env INL_PR_SUBBLOCKS, default 4;
+// 1 = one allgather after the whole gather.
+static int pr_subblocks() {
+  int k = 4;
+  if (const char *e = getenv("INL_PR_SUBBLOCKS")) k = atoi(e);
+  return k < 1 ? 1 : k > 16 ? 16 : k;
 }
 
 void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damping, int iters,
@@ -235,9 +294,15 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
   const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
   const int64_t B = DIST ? (n + P - 1) / P : n;  // row block (inl_partition_rows)
   const int64_t npad = B * P;
-  pr_compact(ctx, p, out_degree, B, DIST ? P : 1);
-  const int64_t Bc = p->pr_bc;                    // compact slots per block (exchange count)
-  const int64_t ncomp = Bc * (DIST ? P : 1) + 1;  // + the zero slot
+  // pipelined exchange: sub-block k's allgather (on the comm stream) overlaps the gathers of
+  // sub-blocks k+1.. (the column-blocked opt-in keeps one launch per iteration)
+  int K = DIST && P > 1 ? pr_subblocks() : 1;
+  if (p->bins.flags & INL_BINS_COLBLOCK) K = 1;
+  pr_compact(ctx, p, out_degree, B, DIST ? P : 1, K);
+  if (p->pr_cb.active) K = 1;
+  const int64_t Bc = p->pr_bc;                        // slots per (rank, sub-block) group
+  const int64_t span = Bc * (DIST ? P : 1);           // slots per sub-block (all ranks)
+  const int64_t ncomp = span * p->pr_K + 1;           // + the zero slot
   float *c_cur = (float *)ctx->s_a.get(sizeof(float) * ncomp);
   float *c_next = (float *)ctx->s_b.get(sizeof(float) * ncomp);
   INL_CUDA(cudaMemsetAsync(c_cur, 0, sizeof(float) * ncomp, st));
@@ -258,21 +323,57 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
 
   const int64_t m = gather_dpart_count(p, &p->pr_cb);
   double *dpart = (double *)p->dpart.p;
+  const int32_t *pr_hot = p->pr_nhot > 0 ? (const int32_t *)p->pr_hot.p : nullptr;
+  cudaStream_t cs = K > 1 ? comm_stream(ctx) : st;
+  // leave SMs to NCCL's kernels while they overlap the gather (the loopback copies use the
+  // copy engines instead)
+  const int max_ctas = K > 1 && ctx->comm ? ctx->num_sms - 16 : 0;
   for (int t = 0; t < iters; ++t) {
     const bool last = t + 1 == iters;
     GatherArgs a{p->row_ptr, p->col_idx, nullptr, c_cur, p->nnz, p->n_rows,
                  p->bins.t_thread, p->bins.t_warp, p->bins.t_block, p->bins.grid_chunk, false};
     PrEpi epi{out_degree, c_next, cidx, last ? (DIST ? rank_pad : rank) : nullptr, base, damping,
               p->row_begin, 0.0f};
-    launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p,
-                         p->pr_nhot > 0 ? (const int32_t *)p->pr_hot.p : nullptr, &p->pr_cb, p->pr_nhot);
-    if (!last) {
-      k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
-      INL_CUDA(cudaGetLastError());
-      if (DIST) {
-        comm_allgather(ctx, c_next + (int64_t)ctx->rank * Bc, c_next, Bc, ncclFloat32, dloc, dall);
+    if (K == 1) {
+      launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p, pr_hot, &p->pr_cb, p->pr_nhot);
+      if (!last) {
+        k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
+        INL_CUDA(cudaGetLastError());
+        if (DIST) comm_allgather(ctx, c_next + (int64_t)ctx->rank * Bc, c_next, Bc, ncclFloat32, dloc, dall);
       }
-      k_pr_base<<<1, 1, 0, st>>>(dall, P, n, (double)damping, base);
+    } else {
+      const WorkItem *items = (const WorkItem *)p->pr_items.p;
+      for (int k = 0; k < K; ++k) {
+        GatherRange rg;
+        rg.items = items + p->pr_iofs[k];
+        rg.n = p->pr_iofs[k + 1] - p->pr_iofs[k];
+        rg.max_ctas = max_ctas;
+        rg.skip_xhot = k > 0;  // x_hot (c_cur's hot slots) is copied once per iteration
+        if (rg.n > 0)
+          launch_gather<false>(ctx, p, a, epi, dpart + p->pr_iofs[k], (const int32_t *)p->pr_col.p, pr_hot, nullptr,
+                               p->pr_nhot, &rg);
+        if (!last) {  // sub-block k's contributions go out while k+1.. are gathered
+          cudaEvent_t ev = ctx_event(ctx, 0);  // a wait captures the record made just before it
+          INL_CUDA(cudaEventRecord(ev, st));
+          INL_CUDA(cudaStreamWaitEvent(cs, ev, 0));
+          float *blk = c_next + (int64_t)k * span;
+          comm_allgather(ctx, blk + (int64_t)ctx->rank * Bc, blk, Bc, ncclFloat32, nullptr, nullptr, cs);
+        }
+      }
+      if (!last) {
+        k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, dloc);
+        INL_CUDA(cudaGetLastError());
+        cudaEvent_t ev = ctx_event(ctx, 1);
+        INL_CUDA(cudaEventRecord(ev, st));
+        INL_CUDA(cudaStreamWaitEvent(cs, ev, 0));
+        comm_allgather(ctx, dloc, dall, 1, ncclFloat64, nullptr, nullptr, cs);
+        cudaEvent_t done = ctx_event(ctx, 2);
+        INL_CUDA(cudaEventRecord(done, cs));
+        INL_CUDA(cudaStreamWaitEvent(st, done, 0));  // the next iteration reads every block
+      }
+    }
+    if (!last) {
+      k_pr_base<<<1, 1, 0, st>>>(dall, DIST ? P : 1, n, (double)damping, base);
       INL_CUDA(cudaGetLastError());
       float *tmp = c_cur;
       c_cur = c_next;

@@ -142,7 +142,12 @@ def test_spmv_float_within_1e5(P):
 
 @pytest.mark.parametrize("P", PS)
 @pytest.mark.parametrize("scale", [12, 18])
-def test_pagerank(P, scale):
+@pytest.mark.parametrize("subblocks", [1, 4, 16])
+def test_pagerank(P, scale, subblocks, monkeypatch):
+    """subblocks = row sub-blocks per rank of the pipelined exchange (pagerank.cu): 1 = one
+    allgather after the gather; 4 (default) and 16 (several empty sub-blocks at scale 12)
+    overlap sub-block k's allgather, on the ctx's comm stream, with the later gathers."""
+    monkeypatch.setenv("INL_PR_SUBBLOCKS", str(subblocks))
     g = inlgen.host_build(scale, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.TRANSPOSE)
     n = g.n_global
     ref = oracle.pagerank(n, g.row_ptr, g.col_idx, g.out_degree, 0.85, 20)
