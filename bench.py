@@ -10,8 +10,12 @@ once, timed separately).  Prints ONE JSON line (rank 0).
 
 Under torchrun (N > 1) every rank owns a row block (inl_partition_rows) of an
 R-MAT graph whose scale grows with log2(N) so per-GPU work stays fixed (weak
-scaling); SpMV needs no collective (x replicated), SSSP/BFS/PageRank use the
-library's NCCL exchange.  Time = max over ranks of CUDA-event time.
+scaling), or, with --strong, of the N = 1 graph (strong scaling: PageRank at
+scale 25 is the north star's >= 5x gate).  SpMV needs no collective for one
+product (x replicated; the headline value), and the line also reports the
+product followed by the allgather of y (inl_spmv_allgather, the form an iterated
+SpMV needs); SSSP/BFS/PageRank use the library's NCCL exchange.  Time = max over
+ranks of CUDA-event time.
 """
 from __future__ import annotations
 
@@ -47,6 +51,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--iterations", type=int, default=20, help="PageRank iterations")
+    ap.add_argument("--strong", action="store_true", help="N > 1: keep the N = 1 graph (strong scaling)")
+    ap.add_argument("--no-context", action="store_true", help="skip the cuSPARSE / OpenMP context lines")
     return ap.parse_args()
 
 
@@ -177,7 +183,8 @@ def run_inl(a):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     scale0 = a.scale or DEFAULT_SCALE[a.op]
-    scale = scale0 + int(round(math.log2(world)))  # weak scaling: fixed rows/nnz per GPU
+    # weak scaling: fixed rows/nnz per GPU; --strong: the same graph at every N
+    scale = scale0 + (0 if a.strong else int(round(math.log2(world))))
     stream = torch.cuda.Stream(local)
     torch.cuda.set_stream(stream)
     ctx = inl.Ctx(local)
@@ -315,6 +322,22 @@ def run_inl(a):
     if a.op in ("spmv", "pagerank"):  # per-step figures -> whole timed region
         units_local *= a.steps
         bytes_local *= a.steps
+    ag = None
+    if a.op == "spmv" and world > 1:  # the product followed by the allgather of y (replicated)
+        yg = torch.empty(A.n_global, device="cuda")
+        for _ in range(max(a.warmup, 1)):
+            inl.spmv_allgather(ctx, A, W["val"], W["x"], yg, plan)
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(a.steps):
+            inl.spmv_allgather(ctx, A, W["val"], W["x"], yg, plan)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ag = float(t.item())
     cnt = torch.tensor([int(units_local), int(bytes_local)], dtype=torch.int64, device="cuda")
     kt = torch.tensor([k_ms], dtype=torch.float64, device="cuda")
     if world > 1:
@@ -332,7 +355,7 @@ def run_inl(a):
         out.update({
             "metric": METRIC, "value": round(gteps, 3), "unit": "GTEPS", "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 5),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32" if a.op in ("spmv", "pagerank") else "u32",
+            "higher_is_better": True, "scaling": "strong" if (a.strong and world > 1) else "weak", "vs_baseline": None, "dtype": "f32" if a.op in ("spmv", "pagerank") else "u32",
             "data": "synthetic (R-MAT A,B,C=.57,.19,.19, Philox seeds graph=1 val=3 x=4 w=2, generated on GPU)",
             "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
                                     "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
@@ -354,8 +377,12 @@ def run_inl(a):
                            "kernel_launches": k_launches, "kernel_ms_per_launch": round(k_ms / max(k_launches, 1), 5),
                            "kernel_share_of_step": round(k_ms / ms, 4),
                            "alg_bytes_per_step_per_gpu": int(bytes_total / world / a.steps),
-                           "traffic": traffic_lookup(a.op, scale)}
+                           "traffic": traffic_lookup(a.op, scale, "_t1" if a.thread_only else "")}
         out["plan"] = info
+        if ag is not None:
+            out["with_allgather"] = {"value": round(units_total / (ag * 1e-3) / 1e9, 3), "unit": "GTEPS",
+                                     "ms_per_step": round(ag / a.steps, 5),
+                                     "what": "inl_spmv_allgather: local product + NCCL allgather of y (replicated)"}
     if a.op == "spmv" and not a.no_e2e:
         e2e = e2e_spmv(a, ctx, g, W, torch, world, rank)
         if rank == 0:
@@ -369,20 +396,92 @@ def run_inl(a):
         out["clocks"] = ck.summary()
         if not a.no_cpu_baseline and world == 1:
             out["cpu_baseline"] = cpu_baseline(a.op, g, W, a, torch)
+            if not a.no_context:
+                ctxl = context_lines(a.op, g, W, a, torch, A)
+                if ctxl:
+                    out["context"] = ctxl
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
 
 
-def traffic_lookup(op, scale):
+def traffic_lookup(op, scale, variant=""):
+    """ncu dram bytes per launch of this op's dominant kernel at this scale (profiles/traffic.json),
+    keyed by op, scale and variant ("" = the default kernels, "_t1" = the thread-only baseline)."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     try:
         d = json.load(open(p))
-        v = d.get(f"{op}_s{scale}")
-        return v
+        return d.get(f"{op}_s{scale}{variant}")
     except Exception:
         return None
+
+
+def host_info():
+    """nproc, CPU model and RAM of the box (the oracle's line records them)."""
+    model, ram = None, None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                ram = round(int(line.split()[1]) / 1024 / 1024, 1)
+                break
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model, "ram_gb": ram}
+
+
+def context_lines(op, g, W, a, torch, A):
+    """Context only: the oracle loops under OpenMP on all host cores (bit-identical
+    to the oracle) and, for SpMV, cuSPARSE's CSR SpMV on the same matrix (a library call, timed
+    with CUDA events).  Neither is the product or the parity reference."""
+    import oracle
+    out = {}
+    rp = g["row_ptr"].cpu().numpy()
+    ci = g["col_idx"].cpu().numpy()
+    try:
+        if op == "spmv":
+            val, x = W["val"].cpu().numpy(), W["x"].cpu().numpy()
+            reps, t0 = 0, time.perf_counter()
+            while reps < 3 or time.perf_counter() - t0 < 3.0:
+                oracle.spmv_par(rp, ci, val, x)
+                reps += 1
+            dt = (time.perf_counter() - t0) / reps
+            out["cpu_parallel"] = {"value": round(len(ci) / dt / 1e9, 4), "unit": "GTEPS", "ms": round(dt * 1e3, 2),
+                                   "cores": oracle.par_threads(), "kind": "oracle loops under OpenMP (orc_par.c)"}
+        elif op == "pagerank":
+            t0 = time.perf_counter()
+            oracle.pagerank_par(g["n_global"], rp, ci, g["out_degree"].cpu().numpy(), 0.85, 2)
+            dt = (time.perf_counter() - t0) / 2
+            out["cpu_parallel"] = {"value": round(len(ci) / dt / 1e9, 4), "unit": "GTEPS",
+                                   "ms_per_iteration": round(dt * 1e3, 2), "cores": oracle.par_threads(),
+                                   "kind": "oracle loops under OpenMP (orc_par.c), 2 iterations"}
+    except Exception as e:  # context only: never fail the bench over it
+        out["cpu_parallel"] = {"error": repr(e)[:200]}
+    if op == "spmv":
+        try:
+            M = torch.sparse_csr_tensor(g["row_ptr"], g["col_idx"].long(), W["val"],
+                                        size=(A.n_rows, A.n_global))
+            for _ in range(3):
+                torch.mv(M, W["x"])
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(10):
+                torch.mv(M, W["x"])
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / 10
+            out["cusparse_spmv"] = {"ms": round(ms, 4), "value": round(len(ci) / (ms * 1e-3) / 1e9, 2),
+                                    "unit": "GTEPS", "what": "torch.mv on a CSR tensor (cuSPARSE SpMV, int64 "
+                                    "indices), same matrix / x, CUDA events, 10 calls; library context only"}
+            del M
+        except Exception as e:
+            out["cusparse_spmv"] = {"error": repr(e)[:200]}
+    return out
 
 
 def e2e_spmv(a, ctx, g, W, torch, world, rank):
@@ -433,14 +532,14 @@ def cpu_baseline(op, g, W, a, torch, budget_s=10.0):
                 break
         dt = time.perf_counter() - t0
         return {"value": round(len(ci) * reps / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                "sample": f"full cfg2 matrix ({len(ci)} nnz) x {reps} repetitions, {dt:.1f} s"}
+                "sample": f"full cfg2 matrix ({len(ci)} nnz) x {reps} repetitions, {dt:.1f} s", **host_info()}
     if op == "pagerank":
         t0 = time.perf_counter()
         it = 2
         oracle.pagerank(g["n_global"], rp, ci, g["out_degree"].cpu().numpy(), 0.85, it)
         dt = time.perf_counter() - t0
         return {"value": round(len(ci) * it / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                "sample": f"{it} PageRank iterations on the full graph ({len(ci)} nnz), {dt:.1f} s"}
+                "sample": f"{it} PageRank iterations on the full graph ({len(ci)} nnz), {dt:.1f} s", **host_info()}
     import inlgen
     src = inlgen.sources(rp, 1)[0]
     t0 = time.perf_counter()
@@ -455,7 +554,7 @@ def cpu_baseline(op, g, W, a, torch, budget_s=10.0):
     dt = time.perf_counter() - t0
     m = int((rp[1:] - rp[:-1])[reached].sum())
     return {"value": round(m / dt / 1e9, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle",
-            "sample": f"1 source ({src}), m_reached={m}, {dt:.1f} s"}
+            "sample": f"1 source ({src}), m_reached={m}, {dt:.1f} s", **host_info()}
 
 
 def run_reference(a):
@@ -468,7 +567,7 @@ def run_reference(a):
     import inlgen
     import oracle
     scale0 = a.scale or DEFAULT_SCALE[a.op]
-    scale = scale0 + int(round(math.log2(max(world, 1))))
+    scale = scale0 + (0 if a.strong else int(round(math.log2(max(world, 1)))))
     # bounded: the host generator builds the graph for small scales; large ones use the GPU twin
     try:
         import torch
@@ -514,14 +613,15 @@ def run_reference(a):
     v = units * a.steps / dt / 1e9
     line = {"impl": "reference", "metric": METRIC, "value": round(v, 5), "unit": "GTEPS", "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(dt / a.steps * 1e3, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64" if a.op in ("spmv", "pagerank") else "int64",
+            "higher_is_better": True, "scaling": "strong" if (a.strong and world > 1) else "weak", "vs_baseline": None, "dtype": "f64" if a.op in ("spmv", "pagerank") else "int64",
             "data": "synthetic (same R-MAT recipe and seeds as the inl arm)",
             "config": {"workload": {"spmv": "cfg2 SpMV fp32 R-MAT", "pagerank": "cfg4 PageRank R-MAT in-CSR",
                                     "sssp": "cfg3 SSSP R-MAT symmetric w in 1..255",
                                     "bfs": "cfg5 BFS R-MAT symmetric",
                                     "bc": "NEXT-3 betweenness R-MAT symmetric (one source per step)"}[a.op],
                        "op": a.op, "scale": scale, "edge_factor": a.edge_factor, "n": int(n), "nnz_total": int(len(ci))},
-            "cpu_baseline": {"value": round(v, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": round(v, 5), "unit": "GTEPS", "cores": 1, "kind": "oracle", "sample": sample,
+                             **host_info()},
             "e2e": {"value": round(v, 5), "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 

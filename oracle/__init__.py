@@ -44,6 +44,50 @@ def _rc(rc, what):
         raise RuntimeError(f"{what} returned {rc}")
 
 
+_par = None
+
+
+def par_lib() -> C.CDLL:
+    """liborc_par.so: orc.c's SpMV / PageRank loops with the outer loop under OpenMP — the
+    "CPU-parallel" context line of SURVEY §8d (bit-identical results; not a parity reference)."""
+    global _par
+    if _par is None:
+        p = os.path.join(_HERE, "liborc_par.so")
+        if not os.path.exists(p):
+            raise RuntimeError(f"{p} missing: run `python scripts/build.py --only oracle`")
+        L = C.CDLL(p)
+        vp, i64 = C.c_void_p, C.c_int64
+        L.orc_spmv_par.argtypes = [i64, vp, vp, vp, vp, vp]
+        L.orc_pagerank_par.argtypes = [i64, vp, vp, vp, C.c_double, C.c_int32, vp]
+        _par = L
+    return _par
+
+
+def par_threads() -> int:
+    return int(par_lib().orc_par_threads())
+
+
+def spmv_par(row_ptr, col_idx, val, x) -> np.ndarray:
+    rp, prp = _a(row_ptr, np.int64)
+    ci, pci = _a(col_idx, np.int32)
+    va, pva = _a(val, np.float32)
+    xx, pxx = _a(x, np.float32)
+    n = len(rp) - 1
+    y = np.empty(n, dtype=np.float64)
+    _rc(par_lib().orc_spmv_par(n, prp, pci, pva, pxx, y.ctypes.data if n else 0), "orc_spmv_par")
+    return y
+
+
+def pagerank_par(n, in_row_ptr, in_col_idx, out_degree, damping=0.85, iterations=20) -> np.ndarray:
+    rp, prp = _a(in_row_ptr, np.int64)
+    ci, pci = _a(in_col_idx, np.int32)
+    od, pod = _a(out_degree, np.int32)
+    r = np.empty(n, dtype=np.float64)
+    _rc(par_lib().orc_pagerank_par(n, prp, pci, pod, damping, iterations, r.ctypes.data if n else 0),
+        "orc_pagerank_par")
+    return r
+
+
 def spmv(row_ptr, col_idx, val, x) -> np.ndarray:
     rp, prp = _a(row_ptr, np.int64)
     ci, pci = _a(col_idx, np.int32)

@@ -56,6 +56,16 @@ def build_oracle(force: bool = False) -> str:
     return out
 
 
+def build_oracle_par(force: bool = False) -> str:
+    """The OpenMP "CPU-parallel" context line (oracle/orc_par.c; bench cpu_baseline only)."""
+    out = os.path.join(ROOT, "oracle", "liborc_par.so")
+    src = os.path.join(ROOT, "oracle", "orc_par.c")
+    if force or _stale(out, [src]):
+        _run(["gcc", "-O2", "-std=c99", "-fPIC", "-shared", "-fopenmp", "-ffp-contract=off", "-fno-fast-math",
+              "-Wall", "-o", out, src])
+    return out
+
+
 def build_inlgen(force: bool = False) -> str:
     out = os.path.join(ROOT, "inlgen", "libinlgen.so")
     d = os.path.join(ROOT, "inlgen")
@@ -93,6 +103,7 @@ def build_all(force: bool = False, only: str | None = None) -> list[str]:
     outs = []
     if only in (None, "oracle"):
         outs.append(build_oracle(force))
+        outs.append(build_oracle_par(force))
     if only in (None, "inlgen"):
         outs.append(build_inlgen(force))
     if only in (None, "inl"):

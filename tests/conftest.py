@@ -25,6 +25,7 @@ def _built():
     import build  # noqa: E402
 
     build.build_oracle()
+    build.build_oracle_par()
     build.build_inlgen()
     import glob
     if glob.glob(os.path.join(ROOT, "paper_conf_icpp_liwb15_b200", "csrc", "*.cu")):

@@ -129,3 +129,11 @@ def test_fixed_point_matches_linear_solve():
             G[:, u] = 1.0 / n
     p = np.linalg.solve(np.eye(n) - d * G, np.full(n, (1 - d) / n))
     np.testing.assert_allclose(r, p, rtol=1e-12)
+
+
+def test_openmp_context_line_is_bit_identical():
+    import inlgen
+    g = inlgen.host_build(13, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.TRANSPOSE)
+    a = oracle.pagerank_par(g.n_global, g.row_ptr, g.col_idx, g.out_degree, 0.85, 20)
+    b = oracle.pagerank(g.n_global, g.row_ptr, g.col_idx, g.out_degree, 0.85, 20)
+    assert np.array_equal(a, b)

@@ -101,3 +101,13 @@ def test_rmat_against_scipy_and_row_sums():
     rs = oracle.spmv(g.row_ptr, g.col_idx, val, ones)
     np.testing.assert_allclose(rs, np.add.reduceat(np.r_[val.astype(np.float64), 0], g.row_ptr[:-1])
                                * (np.diff(g.row_ptr) > 0), rtol=1e-13)
+
+
+def test_openmp_context_line_is_bit_identical():
+    """The "CPU-parallel" context line (oracle/orc_par.c) only splits the row loop."""
+    import inlgen
+    g = inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH)
+    val = inlgen.values_host(g.row_ptr, g.col_idx)
+    x = inlgen.vector_host(g.n_global)
+    assert np.array_equal(oracle.spmv_par(g.row_ptr, g.col_idx, val, x), oracle.spmv(g.row_ptr, g.col_idx, val, x))
+    assert oracle.par_threads() >= 1
