@@ -256,7 +256,8 @@ def run_inl(a):
     # the dominant kernel(s), timed live by the library with events on its own stream
     kernels = (["k_gather", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
                else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
-               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_sssp_split"])
+               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_thread", "k_bu_warp",
+                     "k_sssp_split"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
     ctx.ktimer_enable(True)
@@ -313,7 +314,9 @@ def run_inl(a):
                 r["edges_relaxed"] = 2 * tot_edges // max(len(reached), 1)
         else:
             relax = sum(r["edges_relaxed"] for r in reached)
-            bytes_local = 8 * relax + 16 * sum(r["frontier_total"] for r in reached)
+            # per examined edge: col_idx (+ the weight for SSSP); per frontier vertex: row_ptr pair,
+            # queue entry, distance/level (bitmaps and dist stay L2-resident)
+            bytes_local = (8 if a.op == "sssp" else 4) * relax + 16 * sum(r["frontier_total"] for r in reached)
         if all(r.get("launches", 0) > 0 for r in reached):  # counted by the library
             launches_per_step = sum(r["launches"] for r in reached) / len(reached)
         else:

@@ -116,7 +116,8 @@ typedef struct {
 
 typedef struct {
   int32_t iterations;     /* frontier iterations / BFS levels executed */
-  int64_t edges_relaxed;  /* sum of the degrees of all frontier vertices expanded */
+  int64_t edges_relaxed;  /* edges examined: the degrees of all frontier vertices expanded (top-down /
+                             push steps) + the neighbours read by BFS bottom-up steps */
   int64_t frontier_total; /* sum of frontier sizes over the iterations */
   int64_t launches;       /* kernels the call launched (memsets and copies excluded) */
   int64_t host_syncs;     /* host <-> device round trips of the iteration loop */

@@ -676,6 +676,155 @@ __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *_
   }
 }
 
+// ---- bottom-up with the paper's template: the unvisited vertices of
+// degree > 0 are kept in two worklists by degree — thread-mapped (<= kBuThread neighbours:
+// one lane scans serially, 8 neighbour loads in flight) and warp-mapped (above: the warp
+// scans 64 neighbours per step, early exit on __any_sync) — so no lane idles on a visited
+// vertex and no warp waits on one long serial scan (the T1 form above).  A vertex that
+// finds no parent is carried over to the next level's list (order-preserving within a warp).
+constexpr int kBuThread = 32;
+
+// warp-aggregated, order-preserving (within the warp) append of the lanes with `take`
+__device__ __forceinline__ void push_ballot(int32_t *q, int *cnt, int32_t v, bool take) {
+  const unsigned m = __ballot_sync(0xffffffffu, take);
+  if (!m) return;
+  const int lane = threadIdx.x & 31;
+  int base = 0;
+  if (lane == __ffs(m) - 1) base = atomicAdd(cnt, __popc(m));
+  base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
+  if (take) q[base + __popc(m & ((1u << lane) - 1u))] = v;
+}
+
+// unvisited vertices of degree > 0 -> the thread / warp lists (entering bottom-up)
+__global__ void k_bu_lists(const int64_t *__restrict__ rp, int64_t n, const uint32_t *__restrict__ visited,
+                           int32_t *small, int *ns, int32_t *large, int *nl) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t nn = (n + 31) / 32 * 32;  // whole warps iterate together
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nn; v += stride) {
+    int64_t d = 0;
+    if (v < n && !((visited[v >> 5] >> (v & 31)) & 1u)) d = rp[v + 1] - rp[v];
+    push_ballot(small, ns, (int32_t)v, d > 0 && d <= kBuThread);
+    push_ballot(large, nl, (int32_t)v, d > kBuThread);
+  }
+}
+
+struct BuArgs {
+  const int64_t *rp;
+  const int32_t *col;
+  const uint32_t *fcur;  // current frontier bitmap
+  uint32_t *fnext;       // next frontier bitmap (cleared before the level)
+  uint32_t *visited;
+  int32_t *level;
+  int L;
+  const int32_t *in;     // this level's list
+  int n_in;
+  int32_t *out;          // vertices still without a parent
+  int *n_out;
+  int *found;            // newly visited vertices
+  unsigned long long *mf;  // their degree sum (Beamer's m_f)
+  uint64_t pol;
+  unsigned long long *examined;  // neighbours read (the stats' edges_relaxed)
+};
+
+__device__ __forceinline__ void bu_visit(const BuArgs &a, int32_t v) {
+  const uint32_t bit = 1u << (v & 31);
+  a.level[v] = a.L + 1;
+  atomicOr(a.fnext + (v >> 5), bit);
+  atomicOr(a.visited + (v >> 5), bit);
+}
+
+// thread bin: one lane per vertex, its <= kBuThread neighbours 8 at a time
+__global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
+  a.pol = policy_evict_first();
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t nn = ((int64_t)a.n_in + 31) / 32 * 32;
+  int fcnt = 0;
+  unsigned long long dg = 0, ex = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nn; i += stride) {
+    const bool valid = i < a.n_in;
+    const int32_t v = valid ? a.in[i] : 0;
+    bool found = false;
+    int64_t s = 0, e = 0;
+    if (valid) {
+      s = a.rp[v];
+      e = a.rp[v + 1];
+    }
+    for (int64_t k = s; k < e && !found; k += 8) {
+      ex += (unsigned long long)min((int64_t)8, e - k);
+      int32_t u[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) u[j] = k + j < e ? (int32_t)ld_stream_pol(a.col + k + j, a.pol) : -1;
+      uint32_t fw[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) fw[j] = u[j] >= 0 ? __ldg(a.fcur + (u[j] >> 5)) : 0u;
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        if (u[j] >= 0 && ((fw[j] >> (u[j] & 31)) & 1u)) found = true;
+    }
+    if (found) {
+      bu_visit(a, v);
+      ++fcnt;
+      dg += (unsigned long long)(e - s);
+    }
+    push_ballot(a.out, a.n_out, v, valid && !found);
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    fcnt += __shfl_xor_sync(0xffffffffu, fcnt, o);
+    dg += __shfl_xor_sync(0xffffffffu, dg, o);
+    ex += __shfl_xor_sync(0xffffffffu, ex, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (fcnt) {
+      atomicAdd(a.found, fcnt);
+      atomicAdd(a.mf, dg);
+    }
+    if (ex) atomicAdd(a.examined, ex);
+  }
+}
+
+// warp bin: one warp per vertex, 64 neighbours per step (two loads per lane in flight)
+__global__ void __launch_bounds__(256) k_bu_warp(BuArgs a) {
+  a.pol = policy_evict_first();
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  int fcnt = 0;
+  unsigned long long dg = 0, ex = 0;
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < a.n_in; i += nw) {
+    const int32_t v = a.in[i];
+    const int64_t s = a.rp[v], e = a.rp[v + 1];
+    bool found = false;
+    for (int64_t k = s; k < e; k += 64) {
+      ex += (unsigned long long)min((int64_t)64, e - k);
+      const int64_t k0 = k + lane, k1 = k + 32 + lane;
+      const int32_t u0 = k0 < e ? (int32_t)ld_stream_pol(a.col + k0, a.pol) : -1;
+      const int32_t u1 = k1 < e ? (int32_t)ld_stream_pol(a.col + k1, a.pol) : -1;
+      const uint32_t f0 = u0 >= 0 ? __ldg(a.fcur + (u0 >> 5)) : 0u;
+      const uint32_t f1 = u1 >= 0 ? __ldg(a.fcur + (u1 >> 5)) : 0u;
+      const bool hit = (u0 >= 0 && ((f0 >> (u0 & 31)) & 1u)) || (u1 >= 0 && ((f1 >> (u1 & 31)) & 1u));
+      if (__any_sync(0xffffffffu, hit)) {
+        found = true;
+        break;
+      }
+    }
+    if (lane == 0) {
+      if (found) {
+        bu_visit(a, v);
+        ++fcnt;
+        dg += (unsigned long long)(e - s);
+      } else {
+        a.out[atomicAdd(a.n_out, 1)] = v;
+      }
+    }
+  }
+  if (lane == 0) {
+    if (fcnt) {
+      atomicAdd(a.found, fcnt);
+      atomicAdd(a.mf, dg);
+    }
+    if (ex) atomicAdd(a.examined, ex);
+  }
+}
+
 __global__ void k_queue_to_bitmap(const int32_t *__restrict__ q, int nq, uint32_t *__restrict__ bm) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nq; i += gridDim.x * blockDim.x)
     atomicOr(bm + (q[i] >> 5), 1u << (q[i] & 31));
@@ -1044,9 +1193,26 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
     *mfn = *(volatile unsigned long long *)((int *)ctx->pinned + 10);
     m_u -= (double)*mfn;
   };
+  // binned bottom-up worklists (thread / warp bins, current and next); INL_BFS_BU=word keeps
+  // the one-thread-per-vertex word kernel (measurement switch)
+  static int bu_word = -1;
+  if (bu_word < 0) {
+    const char *e = getenv("INL_BFS_BU");
+    bu_word = e && std::string(e) == "word";
+  }
+  int32_t *bl_s[2] = {nullptr, nullptr}, *bl_l[2] = {nullptr, nullptr};
+  int n_small = 0, n_large = 0, bl_cur = 0;
+  bool lists_ok = false;  // the worklists hold exactly the unvisited vertices of degree > 0
   if (allow_bu) {
     fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
     fb = fa + nwords + 1;
+    if (!bu_word) {
+      int32_t *L4 = (int32_t *)ctx->s_bu.get(sizeof(int32_t) * 4 * (size_t)(n + 1));
+      for (int q = 0; q < 2; ++q) {
+        bl_s[q] = L4 + (size_t)q * (n + 1);
+        bl_l[q] = L4 + (size_t)(2 + q) * (n + 1);
+      }
+    }
   }
   for (;;) {
     ftotal += nF;
@@ -1062,13 +1228,47 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
         }
         INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
-        {
+        if (bu_word) {
           KScope ks(ctx, "k_bfs_bottom_up");
           k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
                                                            f.counts, mfp);
+          INL_CUDA(cudaGetLastError());
+          read_level(&nF, &mf_next);
+        } else {
+          if (!lists_ok) {  // entering bottom-up: the unvisited vertices, binned by degree
+            INL_CUDA(cudaMemsetAsync(f.counts + 4, 0, 2 * sizeof(int), st));
+            k_bu_lists<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(G.row_ptr, n, bm, bl_s[0], f.counts + 4, bl_l[0],
+                                                                  f.counts + 5);
+            INL_CUDA(cudaGetLastError());
+            INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts + 4, 2 * sizeof(int), cudaMemcpyDeviceToHost, st));
+            INL_CUDA(cudaStreamSynchronize(st));
+            n_small = ((volatile int *)ctx->pinned)[0];
+            n_large = ((volatile int *)ctx->pinned)[1];
+            bl_cur = 0;
+            lists_ok = true;
+          }
+          INL_CUDA(cudaMemsetAsync(fb, 0, sizeof(uint32_t) * nwords, st));
+          INL_CUDA(cudaMemsetAsync(f.counts + 6, 0, 2 * sizeof(int), st));
+          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, bl_s[bl_cur ^ 1],
+                    f.counts + 6, f.counts, mfp, 0, f.relaxed};
+          if (n_small > 0) {
+            KScope ks(ctx, "k_bu_thread");
+            k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
+          }
+          ba.in = bl_l[bl_cur];
+          ba.n_in = n_large;
+          ba.out = bl_l[bl_cur ^ 1];
+          ba.n_out = f.counts + 7;
+          if (n_large > 0) {
+            KScope ks(ctx, "k_bu_warp");
+            k_bu_warp<<<grid_for((int64_t)n_large * 32, ctx->num_sms), 256, 0, st>>>(ba);
+          }
+          INL_CUDA(cudaGetLastError());
+          read_level(&nF, &mf_next);
+          n_small = ((volatile int *)ctx->pinned)[6];
+          n_large = ((volatile int *)ctx->pinned)[7];
+          bl_cur ^= 1;
         }
-        INL_CUDA(cudaGetLastError());
-        read_level(&nF, &mf_next);
         std::swap(fa, fb);
         queue_ok = false;
       } else {
@@ -1077,6 +1277,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           k_bitmap_to_queue<<<grid_for(nwords, ctx->num_sms), 256, 0, st>>>(fa, n, f.F, f.counts);
           INL_CUDA(cudaGetLastError());
         }
+        lists_ok = false;  // top-down visits vertices the worklists still hold
         BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, allow_bu ? mfp : nullptr};  // m_f only when it decides
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
         expand(ctx, G, b, f, nF, op);

@@ -143,6 +143,7 @@ struct inl_ctx_s {
   inl::DevBuf h_rp, h_ci, h_val, h_x, h_y, h_w, h_od;  // host-staging device copies
   inl::DevBuf s_loop;                                  // loopback allreduce scratch
   inl::DevBuf s_pad;                                   // padded replicated vectors (P > 1)
+  inl::DevBuf s_bu;                                    // BFS bottom-up worklists
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
