@@ -24,6 +24,10 @@
 #include <cstdlib>
 
 #include <cub/block/block_scan.cuh>
+#include <cub/device/device_partition.cuh>
+#include <cub/device/device_select.cuh>
+#include <thrust/iterator/discard_iterator.h>
+#include <thrust/iterator/counting_iterator.h>
 
 #include "comm.h"
 #include "inl_internal.cuh"
@@ -684,29 +688,23 @@ __global__ void k_bfs_bottom_up(const int64_t *__restrict__ rp, const int32_t *_
 // finds no parent is carried over to the next level's list (order-preserving within a warp).
 constexpr int kBuThread = 32;
 
-// warp-aggregated, order-preserving (within the warp) append of the lanes with `take`
-__device__ __forceinline__ void push_ballot(int32_t *q, int *cnt, int32_t v, bool take) {
-  const unsigned m = __ballot_sync(0xffffffffu, take);
-  if (!m) return;
-  const int lane = threadIdx.x & 31;
-  int base = 0;
-  if (lane == __ffs(m) - 1) base = atomicAdd(cnt, __popc(m));
-  base = __shfl_sync(0xffffffffu, base, __ffs(m) - 1);
-  if (take) q[base + __popc(m & ((1u << lane) - 1u))] = v;
-}
-
-// unvisited vertices of degree > 0 -> the thread / warp lists (entering bottom-up)
-__global__ void k_bu_lists(const int64_t *__restrict__ rp, int64_t n, const uint32_t *__restrict__ visited,
-                           int32_t *small, int *ns, int32_t *large, int *nl) {
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t nn = (n + 31) / 32 * 32;  // whole warps iterate together
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nn; v += stride) {
-    int64_t d = 0;
-    if (v < n && !((visited[v >> 5] >> (v & 31)) & 1u)) d = rp[v + 1] - rp[v];
-    push_ballot(small, ns, (int32_t)v, d > 0 && d <= kBuThread);
-    push_ballot(large, nl, (int32_t)v, d > kBuThread);
+// Worklist maintenance through CUB's decoupled look-back selects (stable, one pass each):
+// a per-warp counter atomic on one address serialises at its L2 slice (measured: 2.7 ms to
+// build the lists at scale 26 that way).
+struct BuBin {  // unvisited, degree in (lo, hi]
+  const int64_t *rp;
+  const uint32_t *visited;
+  int64_t lo, hi;
+  __device__ __forceinline__ bool operator()(int32_t v) const {
+    if ((visited[v >> 5] >> (v & 31)) & 1u) return false;
+    const int64_t d = rp[v + 1] - rp[v];
+    return d > lo && d <= hi;
   }
-}
+};
+struct BuUnvisited {
+  const uint32_t *visited;
+  __device__ __forceinline__ bool operator()(int32_t v) const { return !((visited[v >> 5] >> (v & 31)) & 1u); }
+};
 
 struct BuArgs {
   const int64_t *rp;
@@ -718,8 +716,6 @@ struct BuArgs {
   int L;
   const int32_t *in;     // this level's list
   int n_in;
-  int32_t *out;          // vertices still without a parent
-  int *n_out;
   int *found;            // newly visited vertices
   unsigned long long *mf;  // their degree sum (Beamer's m_f)
   uint64_t pol;
@@ -766,7 +762,6 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
       ++fcnt;
       dg += (unsigned long long)(e - s);
     }
-    push_ballot(a.out, a.n_out, v, valid && !found);
   }
   for (int o = 16; o > 0; o >>= 1) {
     fcnt += __shfl_xor_sync(0xffffffffu, fcnt, o);
@@ -806,14 +801,10 @@ __global__ void __launch_bounds__(256) k_bu_warp(BuArgs a) {
         break;
       }
     }
-    if (lane == 0) {
-      if (found) {
-        bu_visit(a, v);
-        ++fcnt;
-        dg += (unsigned long long)(e - s);
-      } else {
-        a.out[atomicAdd(a.n_out, 1)] = v;
-      }
+    if (lane == 0 && found) {
+      bu_visit(a, v);
+      ++fcnt;
+      dg += (unsigned long long)(e - s);
     }
   }
   if (lane == 0) {
@@ -1236,10 +1227,13 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           read_level(&nF, &mf_next);
         } else {
           if (!lists_ok) {  // entering bottom-up: the unvisited vertices, binned by degree
-            INL_CUDA(cudaMemsetAsync(f.counts + 4, 0, 2 * sizeof(int), st));
-            k_bu_lists<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(G.row_ptr, n, bm, bl_s[0], f.counts + 4, bl_l[0],
-                                                                  f.counts + 5);
-            INL_CUDA(cudaGetLastError());
+            thrust::counting_iterator<int32_t> iota(0);
+            size_t need = 0;
+            const BuBin sm{G.row_ptr, bm, 0, kBuThread}, lg{G.row_ptr, bm, kBuThread, INT64_MAX};
+            thrust::discard_iterator<> none;
+            INL_CUDA(cub::DevicePartition::If(nullptr, need, iota, bl_s[0], bl_l[0], none, f.counts + 4, (int)n, sm, lg, st));
+            INL_CUDA(cub::DevicePartition::If(ctx->s_tmp.get(need), need, iota, bl_s[0], bl_l[0], none, f.counts + 4,
+                                              (int)n, sm, lg, st));
             INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts + 4, 2 * sizeof(int), cudaMemcpyDeviceToHost, st));
             INL_CUDA(cudaStreamSynchronize(st));
             n_small = ((volatile int *)ctx->pinned)[0];
@@ -1249,21 +1243,32 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           }
           INL_CUDA(cudaMemsetAsync(fb, 0, sizeof(uint32_t) * nwords, st));
           INL_CUDA(cudaMemsetAsync(f.counts + 6, 0, 2 * sizeof(int), st));
-          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, bl_s[bl_cur ^ 1],
-                    f.counts + 6, f.counts, mfp, 0, f.relaxed};
+          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, f.counts, mfp, 0, f.relaxed};
           if (n_small > 0) {
             KScope ks(ctx, "k_bu_thread");
             k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
           }
           ba.in = bl_l[bl_cur];
           ba.n_in = n_large;
-          ba.out = bl_l[bl_cur ^ 1];
-          ba.n_out = f.counts + 7;
           if (n_large > 0) {
             KScope ks(ctx, "k_bu_warp");
             k_bu_warp<<<grid_for((int64_t)n_large * 32, ctx->num_sms), 256, 0, st>>>(ba);
           }
           INL_CUDA(cudaGetLastError());
+          // carry the vertices still without a parent over to the next level's lists
+          const BuUnvisited un{bm};
+          if (n_small > 0) {
+            size_t need = 0;
+            INL_CUDA(cub::DeviceSelect::If(nullptr, need, bl_s[bl_cur], bl_s[bl_cur ^ 1], f.counts + 6, n_small, un, st));
+            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, bl_s[bl_cur], bl_s[bl_cur ^ 1], f.counts + 6,
+                                           n_small, un, st));
+          }
+          if (n_large > 0) {
+            size_t need = 0;
+            INL_CUDA(cub::DeviceSelect::If(nullptr, need, bl_l[bl_cur], bl_l[bl_cur ^ 1], f.counts + 7, n_large, un, st));
+            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, bl_l[bl_cur], bl_l[bl_cur ^ 1], f.counts + 7,
+                                           n_large, un, st));
+          }
           read_level(&nF, &mf_next);
           n_small = ((volatile int *)ctx->pinned)[6];
           n_large = ((volatile int *)ctx->pinned)[7];
