@@ -254,7 +254,7 @@ def run_inl(a):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     reached = []
     # the dominant kernel(s), timed live by the library with events on its own stream
-    kernels = (["k_gather", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
+    kernels = (["k_gather", "k_gather_chunks", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
                else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
                else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_thread", "k_bu_warp", "k_bu_deep",
                      "k_sssp_split"])

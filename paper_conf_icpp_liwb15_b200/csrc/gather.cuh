@@ -429,6 +429,129 @@ __global__ void __launch_bounds__(NWARP * 32, 1) k_gather(GatherPlan gp, GatherA
   }
 }
 
+// Long-row pieces alone (the grid / block bins of rows longer than t_warp; dbuf-global,
+// P5@2721).  A piece is part of one row, so there is no row bookkeeping: a warp streams it in
+// passes of 256 entries (lane l: entries 8l..8l+7) with the NEXT pass's columns and values in
+// flight while this pass's gathers run (both double-buffered: this kernel has the registers
+// the tile kernel spends on row tracking), sums the 8 products per lane, chains the pass sums
+// per lane and reduces across the warp once per piece; the last piece of a row (acq_rel
+// ticket) adds the row's partials in piece order in fp64, as k_gather does.  Worst-case
+// rounding depth per piece: 8 + passes + 5 (relative error <= depth * 2^-24 for the
+// non-negative data of the configs).  Runs before k_gather on items [0, n_chunks).
+template <bool VALS, class Epi>
+__global__ void __launch_bounds__(1024, 1) k_gather_chunks(GatherPlan gp, GatherArgs a, Epi epi) {
+  constexpr int E = 8, P = 256;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  float *xs = reinterpret_cast<float *>(smem_raw);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, NWARP = blockDim.x >> 5;
+  const int gw = blockIdx.x * NWARP + warp, nwarps = gridDim.x * NWARP;
+  for (int i = threadIdx.x * 4; i < gp.n_hot; i += blockDim.x * 4)
+    *reinterpret_cast<float4 *>(xs + i) = __ldg(reinterpret_cast<const float4 *>(gp.x_hot + i));
+  if (threadIdx.x == 0) xs[gp.n_hot] = 0.0f;
+  __syncthreads();
+  epi.init();
+  const uint32_t xs_base = smem_u32(xs);
+  const uint32_t ZS = 0x80000000u | (uint32_t)gp.n_hot;
+  const uint64_t pol = 0;
+  if (gw >= gp.n_items) return;
+  auto grab = [&]() -> int {
+    unsigned long long t = 0;
+    if (lane == 0) t = atomicAdd(gp.ticket, 1ull) - gp.base;
+    t = __shfl_sync(0xffffffffu, t, 0);
+    return (int)min(t + (unsigned long long)nwarps, (unsigned long long)gp.n_items);
+  };
+  // columns (resp. values) of entries [k0, k0 + 8) of an item spanning [s, e); outside it the
+  // zero slot (resp. 0)
+  auto load_c = [&](int64_t s, int64_t e, int64_t k0, uint32_t (&cv)[E]) {
+    if (a.vec && k0 >= s && k0 + E <= e) {
+      const U32x8 c = ld_stream_256(a.col_idx + k0);
+#pragma unroll
+      for (int j = 0; j < E; ++j) cv[j] = c.v[j];
+    } else {
+#pragma unroll
+      for (int j = 0; j < E; ++j) {
+        const bool in = k0 + j >= s && k0 + j < e;
+        const uint32_t c = ld_stream_pred(a.col_idx + k0 + j, in);
+        cv[j] = in ? c : ZS;
+      }
+    }
+  };
+  auto load_v = [&](int64_t s, int64_t e, int64_t k0, float (&v)[E]) {
+    if (a.vec && k0 >= s && k0 + E <= e) {
+      const U32x8 w = ld_stream_256(a.val + k0);
+#pragma unroll
+      for (int j = 0; j < E; ++j) v[j] = __uint_as_float(w.v[j]);
+    } else {
+#pragma unroll
+      for (int j = 0; j < E; ++j) {
+        const bool in = k0 + j >= s && k0 + j < e;
+        const float x = __uint_as_float(ld_stream_pred(a.val + k0 + j, in));
+        v[j] = in ? x : 0.0f;
+      }
+    }
+  };
+  int idx = gw;
+  int64_t is = gp.items[idx].s, ie = gp.items[idx].e;  // the rest of the descriptor is re-read at the end
+  uint32_t cv[E];
+  load_c(is, ie, (is & ~(int64_t)(E - 1)) + E * lane, cv);
+  for (;;) {
+    const int nidx = grab();
+    const bool has_next = nidx < gp.n_items;
+    int64_t ns = 0, ne = 0;
+    if (has_next) {
+      ns = gp.items[nidx].s;
+      ne = gp.items[nidx].e;
+    }
+    const int64_t a0 = is & ~(int64_t)(E - 1);
+    float acc = 0.0f;
+    for (int64_t kb = a0;; kb += P) {
+      // this pass's values (in flight with its gathers), the next pass's columns
+      float vv[E];
+      if (VALS) load_v(is, ie, kb + E * lane, vv);
+      uint32_t cn[E];
+      const bool more = kb + P < ie;
+      if (more) load_c(is, ie, kb + P + E * lane, cn);
+      else if (has_next) load_c(ns, ne, (ns & ~(int64_t)(E - 1)) + E * lane, cn);
+      float ps = 0.0f;
+#pragma unroll
+      for (int j = 0; j < E; ++j) {
+        const float xv = gx((int32_t)cv[j], xs_base, a.x, pol);
+        ps += VALS ? vv[j] * xv : xv;
+      }
+      acc += ps;
+#pragma unroll
+      for (int j = 0; j < E; ++j) cv[j] = cn[j];
+      if (!more) break;
+    }
+    const float tot = warp_sum(acc);
+    if (lane == 0) {
+      const WorkItem it = gp.items[idx];
+      double dacc = 0.0;
+      if (it.nch == 1) {
+        dacc = epi(it.r0, tot);
+      } else {
+        gp.partials[it.pbase + it.c] = tot;
+        cuda::atomic_ref<int, cuda::thread_scope_device> tk(gp.tickets[it.j]);
+        if (tk.fetch_add(1, cuda::memory_order_acq_rel) == it.nch - 1) {
+          double t = 0.0;  // partials combined in piece order, fp64 accumulator
+          for (int q = 0; q < it.nch; ++q) {
+            cuda::atomic_ref<float, cuda::thread_scope_device> pq(gp.partials[it.pbase + q]);
+            t += (double)pq.load(cuda::memory_order_relaxed);
+          }
+          dacc = epi(it.r0, (float)t);
+          tk.store(0, cuda::memory_order_relaxed);
+        }
+      }
+      if (Epi::kDangling) gp.dpart[idx] = dacc;
+    }
+    __syncwarp();
+    if (!has_next) break;
+    idx = nidx;
+    is = ns;
+    ie = ne;
+  }
+}
+
 // The paper's baseline (T1, P3@9322, P5@14490): one thread per row, serial inner
 // loop, no load balancing.  Used only as the in-build comparator.
 template <class Epi>
@@ -462,6 +585,39 @@ void launch_gather_t(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, con
   if (grid > need) grid = need;
   KScope ks(ctx, "k_gather");
   kern<<<(int)grid, NWARP * 32, smem, ctx->stream>>>(gp, a, epi);
+  INL_CUDA(cudaGetLastError());
+}
+
+// INL_GATHER_SPLIT=1 (opt-in experiment): long-row pieces in k_gather_chunks, then the tiles in
+// k_gather.  Default 0: every item in k_gather.  Measured at scale 22 (profiles/r02/
+// spmv_chunk_split.txt): 74-91 us for the pieces + 134 us for the tiles vs 185-188 us for the
+// fused kernel — both kernels gather at the same ~310 G entries/s, the L1TEX wavefront rate of
+// the x gathers, so removing the row bookkeeping from the pieces buys nothing and the split
+// loses the fused kernel's overlap of long and short items.
+inline int gather_split() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("INL_GATHER_SPLIT");
+    v = e ? atoi(e) != 0 : 0;
+  }
+  return v;
+}
+
+template <bool VALS, class Epi>
+void launch_gather_chunks(inl_ctx ctx, const GatherPlan &gp, const GatherArgs &a, const Epi &epi) {
+  const size_t smem = (size_t)gp.n_hot * 4 + 16;
+  auto kern = k_gather_chunks<VALS, Epi>;
+  static size_t configured[kMaxDevices] = {};
+  size_t &cf = configured[ctx->device % kMaxDevices];
+  if (smem > cf) {
+    INL_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cf = smem;
+  }
+  int64_t grid = ctx->num_sms;
+  const int64_t need = (gp.n_items + 31) / 32;
+  if (grid > need) grid = need;
+  KScope ks(ctx, "k_gather_chunks");
+  kern<<<(int)grid, 1024, smem, ctx->stream>>>(gp, a, epi);
   INL_CUDA(cudaGetLastError());
 }
 
@@ -521,9 +677,21 @@ void launch_gather(inl_ctx ctx, inl_plan p, const GatherArgs &a_in, const Epi &e
     static int w24 = -1;
     if (w24 < 0) w24 = getenv("INL_GATHER_W24") ? 1 : 0;
     const int mc = ranged ? range->max_ctas : 0;
-    if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi, mc);
-    else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi, mc);
-    else launch_gather_t<8, VALS>(ctx, gp, a, epi, mc);
+    const int64_t n_split = (!ranged && !use_cb && gather_split()) ? p->n_chunks : 0;
+    if (n_split > 0) {  // long-row pieces first, in their own kernel (items [0, n_chunks))
+      GatherPlan gc = gp;
+      gc.n_items = (int)n_split;
+      launch_gather_chunks<VALS>(ctx, gc, a, epi);
+      gp.items += n_split;
+      gp.n_items -= (int)n_split;
+      if (gp.dpart) gp.dpart += n_split;
+      gp.base += (unsigned long long)n_split;
+    }
+    if (gp.n_items > 0) {
+      if (gather_entries_per_lane() == 16) launch_gather_t<16, VALS>(ctx, gp, a, epi, mc);
+      else if (w24) launch_gather_t<8, VALS, Epi, 24>(ctx, gp, a, epi, mc);
+      else launch_gather_t<8, VALS>(ctx, gp, a, epi, mc);
+    }
     p->ticket_base += (unsigned long long)n_items;  // only once the launch was accepted
   }
   if (use_cb && !ranged) launch_cb<VALS>(ctx, *cb, a_in.val, a_in.x, epi, dpart ? dpart + n_items : nullptr);
