@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--bins", type=str, default="", help="t_thread,t_warp,t_block,grid_chunk,cta")
     ap.add_argument("--thread-only", action="store_true", help="paper baseline T1 (no load balancing)")
     ap.add_argument("--colblock", action="store_true", help="long rows column-blocked (INL_BINS_COLBLOCK)")
+    ap.add_argument("--bin-flags", type=int, default=0, help="extra inl_bins.flags (e.g. 4 = INL_BINS_SSSP_DEVLOOP)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--iterations", type=int, default=20, help="PageRank iterations")
@@ -196,7 +197,7 @@ def run_inl(a):
     A = inl.Csr(g["row_ptr"], g["col_idx"], g["n_global"], g["row_begin"])
     bargs = [int(v) for v in a.bins.split(",")] if a.bins else []
     bb = inl.bins(*bargs, flags=(inl.BINS_THREAD_ONLY if a.thread_only else 0) |
-                  (inl.BINS_COLBLOCK if a.colblock else 0))
+                  (inl.BINS_COLBLOCK if a.colblock else 0) | a.bin_flags)
     t0 = time.perf_counter()
     plan = inl.Plan(ctx, A, bb)
     torch.cuda.synchronize()
@@ -257,7 +258,7 @@ def run_inl(a):
     kernels = (["k_gather", "k_gather_chunks", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
                else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
                else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_thread", "k_bu_warp", "k_bu_deep",
-                     "k_sssp_split"])
+                     "k_sssp_split", "sssp_graph"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
     ctx.ktimer_enable(True)

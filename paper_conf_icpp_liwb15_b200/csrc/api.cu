@@ -395,6 +395,7 @@ static void free_ctx(inl_ctx ctx) {
   }
   for (cudaEvent_t e : ctx->events)
     if (e) cudaEventDestroy(e);
+  if (ctx->sssp_graph) sssp_graph_free(ctx->sssp_graph);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
   delete ctx->tplan;
   delete ctx;  // DevBuf destructors free device scratch

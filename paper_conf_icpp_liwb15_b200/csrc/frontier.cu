@@ -20,6 +20,7 @@
 #include <cooperative_groups.h>
 #include <algorithm>
 #include <cstdio>
+#include <cstring>
 #include <string>
 #include <cstdlib>
 
@@ -225,7 +226,7 @@ struct __align__(16) SsspDev {
   int iter, done;
   uint32_t thr, delta;
   int slice;    // dynamic slice counter of k_expand_flat
-  int pad;
+  int pad;      // steps run (k_sssp_post); done = 2 if it ever exceeds kSsspMaxSteps
   unsigned long long ftotal;
 };
 struct SsspDyn {
@@ -573,9 +574,15 @@ __global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) {
   }
 }
 
-// Device-driven step, part 4: roll the state over to the next step.
-__global__ void k_sssp_post(SsspDyn dy) {
+// Device-driven step, part 4: roll the state over to the next step.  In the CUDA-graph loop
+// (a conditional WHILE node around the four kernels) it also sets the loop condition; a step
+// count far beyond any converging run (kSsspMaxSteps) stops the loop with an error flag
+// instead of letting a bug spin the GPU.
+constexpr int kSsspMaxSteps = 1 << 20;
+__global__ void k_sssp_post(SsspDyn dy, cudaGraphConditionalHandle cond, int use_cond) {
   SsspDev *s = dy.s;
+  if (!s->done && ++s->pad > kSsspMaxSteps) s->done = 2;
+  if (use_cond) cudaGraphSetConditional(cond, s->done ? 0u : 1u);
   if (s->done) return;
   const bool split = s->nF == 0;
   if (split) {
@@ -1081,7 +1088,7 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
         KScope ks(ctx, "k_expand_grid");
         k_expand_grid<SsspOp><<<ggrid, NT, 0, st>>>(a, op);
       }
-      k_sssp_post<<<1, 1, 0, st>>>(dy);
+      k_sssp_post<<<1, 1, 0, st>>>(dy, 0, 0);
       launches += 4;
     }
     INL_CUDA(cudaGetLastError());
@@ -1104,6 +1111,139 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   }
 }
 
+// One GPU, near-far, CUDA graph: the step (k_sssp_split, k_expand_flat, k_expand_grid,
+// k_sssp_post) is the body of a conditional WHILE node that k_sssp_post keeps enabled until
+// the near frontier and the far pile are both empty — the whole source runs as ONE graph
+// launch with no host round trip (host_syncs = 1: the final stats read).  The executable
+// graph is cached in the ctx and rebuilt only when an argument it captured changes.
+struct SsspGraphKey {
+  const int64_t *rp;
+  const int32_t *col;
+  const uint32_t *w;
+  uint32_t *dist;
+  void *bufs[6];
+  int64_t n, nnz, gcap;
+  int t_warp, chunk, gm0, gm1, gm2;
+  uint32_t delta;
+  bool operator==(const SsspGraphKey &o) const { return memcmp(this, &o, sizeof(*this)) == 0; }
+};
+
+struct SsspGraph {
+  SsspGraphKey key{};
+  cudaGraphExec_t exec = nullptr;
+  cudaGraph_t graph = nullptr;
+  ~SsspGraph() {
+    if (exec) cudaGraphExecDestroy(exec);
+    if (graph) cudaGraphDestroy(graph);
+  }
+};
+
+void sssp_graph_free(void *g) { delete static_cast<SsspGraph *>(g); }
+
+static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
+                           uint32_t *dist, inl_stats *stats) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = G.n_global;
+  FrontierBufs f = frontier_bufs(ctx, G, b);
+  INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
+  const int64_t nwb = (n + 31) / 32 + 1;
+  SsspDyn dy;
+  uint32_t *bits = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 3 * nwb);
+  dy.inq[0] = bits;
+  dy.inq[1] = bits + nwb;
+  dy.keep = bits + 2 * nwb;
+  INL_CUDA(cudaMemsetAsync(bits, 0, sizeof(uint32_t) * 3 * nwb, st));
+  dy.far[0] = (int32_t *)ctx->s_g.get(sizeof(int32_t) * (2 * n + 16));
+  dy.far[1] = dy.far[0] + n + 8;
+  dy.buf[0] = f.F;
+  dy.buf[1] = f.Fout;
+  dy.s = (SsspDev *)ctx->s_e.get(sizeof(SsspDev));
+  const bool owned = source >= G.row_begin && source < G.row_begin + G.n_rows;
+  SsspDev h{};
+  h.nF = owned ? 1 : 0;
+  h.thr = h.delta = sssp_delta();
+  INL_CUDA(cudaMemcpyAsync(dy.s, &h, sizeof h, cudaMemcpyHostToDevice, st));
+  const int32_t s0 = (int32_t)(owned ? source - G.row_begin : 0);
+  INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(dist, n, source);
+  INL_CUDA(cudaGetLastError());
+  const ExpandCfg c = expand_cfg(G, b);
+  ExpandArgs a{f.F, 0, G.row_ptr, G.col_idx, c.t_thread, c.t_warp, c.t_block, c.chunk,
+               f.gitems, nullptr, (int)f.gcap, f.counts + 2, f.Fout, nullptr, f.relaxed};
+  a.dyn = dy;
+  SsspOp op{dist, w, nullptr, nullptr, 0, 0, true, 0, 0, nullptr, nullptr, nullptr};
+  static int gm[3] = {2, 8, 2};
+  static bool gm_read = false;
+  if (!gm_read) {
+    gm_read = true;
+    if (const char *e = getenv("INL_SSSP_GRIDS")) sscanf(e, "%d,%d,%d", &gm[0], &gm[1], &gm[2]);
+  }
+  SsspGraphKey key{};
+  key.rp = G.row_ptr;
+  key.col = G.col_idx;
+  key.w = w;
+  key.dist = dist;
+  void *bufs[6] = {dy.s, dy.far[0], bits, f.F, f.Fout, f.gitems};
+  memcpy(key.bufs, bufs, sizeof bufs);
+  key.n = n;
+  key.nnz = G.nnz;
+  key.gcap = f.gcap;
+  key.t_warp = c.t_warp;
+  key.chunk = c.chunk;
+  key.gm0 = gm[0];
+  key.gm1 = gm[1];
+  key.gm2 = gm[2];
+  key.delta = h.delta;
+  SsspGraph *sg = static_cast<SsspGraph *>(ctx->sssp_graph);
+  if (!sg || !(sg->key == key)) {
+    delete sg;
+    ctx->sssp_graph = sg = new SsspGraph();
+    sg->key = key;
+    INL_CUDA(cudaGraphCreate(&sg->graph, 0));
+    cudaGraphConditionalHandle cond;
+    INL_CUDA(cudaGraphConditionalHandleCreate(&cond, sg->graph, 1, cudaGraphCondAssignDefault));
+    cudaGraphNodeParams cp{};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = cond;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    cudaGraphNode_t node;
+    INL_CUDA(cudaGraphAddNode(&node, sg->graph, nullptr, 0, &cp));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+    // the body: captured from the ctx stream into the conditional node's graph
+    INL_CUDA(cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
+    const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
+    k_sssp_split<<<gsplit, 256, 0, st>>>(dy, dist);
+    k_expand_flat<SsspOp><<<gflat, NT, 0, st>>>(a, op);
+    k_expand_grid<SsspOp><<<ggrid, NT, 0, st>>>(a, op);
+    k_sssp_post<<<1, 1, 0, st>>>(dy, cond, 1);
+    cudaGraph_t captured = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(st, &captured);
+    INL_CUDA(ce);
+    INL_CUDA(cudaGraphInstantiate(&sg->exec, sg->graph, 0));
+  }
+  {
+    KScope ks(ctx, "sssp_graph");
+    INL_CUDA(cudaGraphLaunch(sg->exec, st));
+  }
+  SsspDev *hs = (SsspDev *)ctx->pinned;
+  INL_CUDA(cudaMemcpyAsync(hs, dy.s, sizeof(SsspDev), cudaMemcpyDeviceToHost, st));
+  INL_CUDA(cudaStreamSynchronize(st));
+  if (((volatile SsspDev *)hs)->done == 2)
+    raise(INL_ERR_INTERNAL, "sssp graph loop exceeded its step bound");
+  check_overflow(ctx, f);
+  if (stats) {
+    unsigned long long r = 0;
+    INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+    stats->iterations = hs->iter;
+    stats->edges_relaxed = (int64_t)r;
+    stats->frontier_total = (int64_t)hs->ftotal;
+    stats->launches = 1 + 4LL * hs->pad;  // init + 4 kernels per step (one graph launch)
+    stats->host_syncs = 1;
+  }
+}
+
 void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
               uint32_t *dist, inl_stats *stats) {
   cudaStream_t st = ctx->stream;
@@ -1113,9 +1253,15 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   // source for the host-driven one (profiles/r01/sssp_devloop.txt) — its 4 launches per
   // step cost more than the ~40 host round trips they save
   const bool devloop = (b.flags & INL_BINS_SSSP_DEVLOOP) != 0;
+  static int use_graph = -1;  // INL_SSSP_GRAPH=0: the device loop with host polling (r01)
+  if (use_graph < 0) {
+    const char *e = getenv("INL_SSSP_GRAPH");
+    use_graph = e ? atoi(e) != 0 : 1;
+  }
   if (!DIST && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && devloop && sssp_delta() != 0xFFFFFFFFu &&
       n > 0) {
-    sssp_run_dyn(ctx, G, b, w, source, dist, stats);
+    if (use_graph) sssp_run_graph(ctx, G, b, w, source, dist, stats);
+    else sssp_run_dyn(ctx, G, b, w, source, dist, stats);
     return;
   }
   FrontierBufs f = frontier_bufs(ctx, G, b);

@@ -137,6 +137,7 @@ struct inl_ctx_s {
   inl::LoopGroup *loop = nullptr;  // loopback group (inl_comm_init_loopback) instead of NCCL
   cudaStream_t comm_stream = nullptr;  // second stream: exchanges overlapped with the gather
   cudaEvent_t events[inl::kCtxEvents] = {};
+  void *sssp_graph = nullptr;  // cached executable graph of the one-GPU SSSP loop (frontier.cu)
   int nranks = 1, rank = 0;
   // scratch
   inl::DevBuf s_tmp, s_a, s_b, s_c, s_d, s_e, s_f, s_g;
@@ -244,4 +245,5 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
             inl_stats *stats, bool symmetric);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);
+void sssp_graph_free(void *g);  // frontier.cu
 }  // namespace inl
