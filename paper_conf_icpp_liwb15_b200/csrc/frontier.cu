@@ -1210,15 +1210,25 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     cudaGraphNode_t node;
     INL_CUDA(cudaGraphAddNode(&node, sg->graph, nullptr, 0, &cp));
     cudaGraph_t body = cp.conditional.phGraph_out[0];
-    // the body: captured from the ctx stream into the conditional node's graph
-    INL_CUDA(cudaStreamBeginCaptureToGraph(st, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
-    const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
-    k_sssp_split<<<gsplit, 256, 0, st>>>(dy, dist);
-    k_expand_flat<SsspOp><<<gflat, NT, 0, st>>>(a, op);
-    k_expand_grid<SsspOp><<<ggrid, NT, 0, st>>>(a, op);
-    k_sssp_post<<<1, 1, 0, st>>>(dy, cond, 1);
-    cudaGraph_t captured = nullptr;
-    const cudaError_t ce = cudaStreamEndCapture(st, &captured);
+    // the body: captured into the conditional node's graph on a private stream (the ctx
+    // stream may be the legacy default stream, which cannot capture); it runs on the ctx stream
+    cudaStream_t cap = nullptr;
+    INL_CUDA(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+    cudaError_t ce = cudaStreamBeginCaptureToGraph(cap, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
+    if (ce == cudaSuccess) {
+      const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
+      k_sssp_split<<<gsplit, 256, 0, cap>>>(dy, dist);
+      k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
+      k_expand_grid<SsspOp><<<ggrid, NT, 0, cap>>>(a, op);
+      k_sssp_post<<<1, 1, 0, cap>>>(dy, cond, 1);
+      cudaGraph_t captured = nullptr;
+      ce = cudaStreamEndCapture(cap, &captured);
+    }
+    cudaStreamDestroy(cap);
+    if (ce != cudaSuccess) {
+      ctx->sssp_graph = nullptr;
+      delete sg;
+    }
     INL_CUDA(ce);
     INL_CUDA(cudaGraphInstantiate(&sg->exec, sg->graph, 0));
   }
