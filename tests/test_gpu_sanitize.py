@@ -18,7 +18,13 @@ def test_compute_sanitizer(tool):
     if tool == "memcheck":
         cmd += ["--leak-check", "no"]
     cmd += [sys.executable, os.path.join(HERE, "sanitize_driver.py")]
-    p = subprocess.run(cmd, capture_output=True, text=True, timeout=900)
+    env = dict(os.environ)
+    if tool == "racecheck":
+        # racecheck (CUDA 12.9) crashes the process on a graph with a conditional WHILE node
+        # (profiles/r02/sanitize_racecheck_graph.txt); the SSSP device loop's kernels run
+        # under it through the stream-launched loop instead (same kernels, INL_SSSP_GRAPH=0)
+        env["INL_SSSP_GRAPH"] = "0"
+    p = subprocess.run(cmd, capture_output=True, text=True, timeout=900, env=env)
     out = p.stdout + p.stderr
     assert p.returncode == 0, out[-4000:]
     assert "sanitize driver ok" in out
