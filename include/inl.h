@@ -85,8 +85,10 @@ typedef struct {
  * bench configs) processes SpMV/PR rows of degree > max(t_warp,
  * 4 * column blocks) column-blocked: a CTA holds one block of x in shared memory and
  * sums the row's entries in that block (one partial per (row, block) run, combined in
- * block order).  INL_BINS_SSSP_DEVLOOP (opt-in, one GPU): the SSSP near-far step loop
- * runs on the device, the host checks termination every few steps.  At most one
+ * block order).  SSSP on one GPU runs its near-far step loop on the device as ONE CUDA-graph
+ * launch per source (a conditional WHILE node; one host round trip per call);
+ * INL_BINS_SSSP_DEVLOOP keeps that device loop even when the environment variable
+ * INL_SSSP_LOOP=host selects the host-driven loop (measurement switch).  At most one
  * INL_BINS_TPL_* flag, and none combined with another flag (else INL_ERR_INVALID_ARGUMENT
  * from inl_plan_create). */
 enum {
@@ -214,7 +216,7 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
                         int32_t iterations, float *rank, inl_plan plan);
 
 /* SSSP (P5@10241, P11@2218): frontier Bellman-Ford relaxation (atomicMin) until
- * no distance changes.  w [nnz] uint32 >= 1, dist [n_global] uint32 with
+ * no distance changes (one GPU: near-far scheduled, the step loop as one CUDA-graph launch).  w [nnz] uint32 >= 1, dist [n_global] uint32 with
  * UINT32_MAX = unreachable (replicated).  Distances must stay < 2^32 - 2^8.
  * Blocks until converged. */
 inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source,

@@ -1259,19 +1259,18 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
-  // the device-driven loop (sssp_run_dyn) is opt-in: measured 8.5 ms vs 8.0 ms per scale-23
-  // source for the host-driven one (profiles/r01/sssp_devloop.txt) — its 4 launches per
-  // step cost more than the ~40 host round trips they save
-  const bool devloop = (b.flags & INL_BINS_SSSP_DEVLOOP) != 0;
-  static int use_graph = -1;  // INL_SSSP_GRAPH=0: the device loop with host polling (r01)
-  if (use_graph < 0) {
-    const char *e = getenv("INL_SSSP_GRAPH");
-    use_graph = e ? atoi(e) != 0 : 1;
-  }
-  if (!DIST && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && devloop && sssp_delta() != 0xFFFFFFFFu &&
+  // One GPU, near-far: by default the whole step loop is ONE CUDA-graph launch (sssp_run_graph,
+  // 7.40 vs 7.84 ms per scale-23 source for the host-driven loop, profiles/r02/sssp_loops.txt).
+  // INL_SSSP_LOOP=host (the r01 default: one host round trip per step) or =dyn (device loop,
+  // host polling every 4-16 steps) select the others for measurement; INL_BINS_SSSP_DEVLOOP
+  // forces a device loop even then.
+  const char *lp = getenv("INL_SSSP_LOOP");
+  const bool host_loop = lp && std::string(lp) == "host" && !(b.flags & INL_BINS_SSSP_DEVLOOP);
+  const bool dyn_loop = lp && std::string(lp) == "dyn";
+  if (!DIST && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && !host_loop && sssp_delta() != 0xFFFFFFFFu &&
       n > 0) {
-    if (use_graph) sssp_run_graph(ctx, G, b, w, source, dist, stats);
-    else sssp_run_dyn(ctx, G, b, w, source, dist, stats);
+    if (dyn_loop) sssp_run_dyn(ctx, G, b, w, source, dist, stats);
+    else sssp_run_graph(ctx, G, b, w, source, dist, stats);
     return;
   }
   FrontierBufs f = frontier_bufs(ctx, G, b);

@@ -53,8 +53,10 @@ BINS = [None, dict(t_thread=-1, t_warp=32, t_block=128, grid_chunk=64),
         dict(t_thread=1, t_warp=32, t_block=128, grid_chunk=64, flags=inl.BINS_SSSP_DEVLOOP)]
 
 
+@pytest.mark.parametrize("loop", ["graph", "host"])
 @pytest.mark.parametrize("bi", range(len(BINS)))
-def test_cfg1_all_sources_bit_exact(ctx, cfg1, bi):
+def test_cfg1_all_sources_bit_exact(ctx, cfg1, bi, loop, monkeypatch):
+    monkeypatch.setenv("INL_SSSP_LOOP", loop)
     g, w = cfg1
     b = inl.bins(**BINS[bi]) if BINS[bi] is not None else None
     for s in inlgen.sources(g.row_ptr, 8):
@@ -85,7 +87,11 @@ def test_small_graph_edge_cases(ctx):
         assert np.array_equal(lv, oracle.bfs(rp, ci, s))
 
 
-def test_devloop_edge_cases_and_certificate(ctx):
+@pytest.mark.parametrize("loop", ["graph", "dyn"])
+def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch):
+    """The device-driven near-far loop: one CUDA-graph launch per source (default) or
+    stream launches with host polling (INL_SSSP_LOOP=dyn), vs the host-driven loop."""
+    monkeypatch.setenv("INL_SSSP_LOOP", loop)
     b = inl.bins(flags=inl.BINS_SSSP_DEVLOOP)
     rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3), (3, 1)], [5, 6, 7], symmetric=True)
     d, st = gpu_sssp(ctx, rp, ci, w, 6, 0, b)  # isolated source
@@ -101,9 +107,13 @@ def test_devloop_edge_cases_and_certificate(ctx):
     for s in inlgen.sources(g.row_ptr, 3):
         d, st = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, b)
         assert certify_sssp(g.row_ptr, g.col_idx, w, s, d) is None
+        monkeypatch.setenv("INL_SSSP_LOOP", "host")
         ref, st0 = gpu_sssp(ctx, g.row_ptr, g.col_idx, w, g.n_global, s, inl.bins())
+        monkeypatch.setenv("INL_SSSP_LOOP", loop)
         assert np.array_equal(d, ref)
         assert st["launches"] > 0 and st["host_syncs"] < st0["host_syncs"]
+        if loop == "graph":
+            assert st["host_syncs"] == 1
 
 
 def test_host_buffers(ctx, cfg1):
