@@ -56,6 +56,32 @@ int inlgen_graph_export(inlgen_graph g, int64_t *row_ptr, int32_t *col_idx, int3
                         void *stream);
 void inlgen_graph_free(inlgen_graph g);
 
+/* ---- loaders and the CiteSeer-shaped generator: host graphs ---- */
+/* MatrixMarket coordinate file (real / integer / pattern; general / symmetric; 1-based):
+ * self-loops dropped, repeated (row, col) pairs merged keeping the FIRST value, columns sorted.
+ * flags: INLGEN_SYMMETRIC adds (v,u) for every (u,v); INLGEN_TRANSPOSE stores the in-edge CSR
+ * + out_degree (both need a square matrix).  Values (non-pattern files) via
+ * inlgen_graph_values.  Returns 0, -1 bad argument, -2 out of memory, -3 file / format error. */
+int inlgen_load_mtx(const char *path, int flags, inlgen_graph *out);
+/* .inlcsr binary file (little-endian): 8-byte magic "INLCSR\0\1"; int64 n_global, n_rows,
+ * row_begin, nnz, flags (1: values follow, 2: out_degree follows); int64 row_ptr[n_rows+1];
+ * int32 col_idx[nnz]; [float val[nnz]]; [int32 out_degree[n_global]].  Loading checks the
+ * structure (row_ptr[0] = 0, non-decreasing, = nnz at the end, columns in range). */
+int inlgen_save_csr(const char *path, inlgen_graph g);
+int inlgen_load_csr(const char *path, inlgen_graph *out);
+/* A host graph from caller arrays (copied; val / out_degree may be NULL). */
+int inlgen_graph_from_csr(int64_t n_global, int64_t n_rows, int64_t row_begin, const int64_t *row_ptr,
+                          const int32_t *col_idx, const float *val, const int32_t *out_degree,
+                          inlgen_graph *out);
+int inlgen_graph_values(inlgen_graph g, float *val); /* -1 if the graph has none */
+/* Undirected configuration-model graph on n vertices whose degree sequence follows a discrete
+ * truncated power law on [dmin, dmax] with the given mean (exponent solved by bisection);
+ * stubs paired by a Philox-keyed shuffle; both directions stored, self-loops and repeated
+ * pairs removed (so realised degrees can be slightly lower).  The CiteSeer shape of PAPER.md
+ * P5@12491-13052: n = 434102, dmin = 1, dmax = 1188, mean 73.9 (~32.1 M CSR entries). */
+int inlgen_powerlaw_build(int64_t n, int dmin, int dmax, double mean, uint64_t seed, int flags,
+                          inlgen_graph *out);
+
 /* Per-entry inputs for a (local) CSR whose row 0 is global row `row_begin`.
  * *_host: host arrays.  *_dev: device arrays, asynchronous on `stream`. */
 int inlgen_weights_host(int64_t n_rows, int64_t row_begin, const int64_t *row_ptr,

@@ -46,6 +46,12 @@ def lib() -> C.CDLL:
         for nm in ("inlgen_values_host", "inlgen_values_dev"):
             getattr(L, nm).argtypes = [i64, i64, vp, vp, u64, i32, vp] + ([vp] if nm.endswith("dev") else [])
         L.inlgen_vector_host.argtypes = [i64, i64, u64, i32, vp]
+        L.inlgen_load_mtx.argtypes = [C.c_char_p, i32, C.POINTER(vp)]
+        L.inlgen_save_csr.argtypes = [C.c_char_p, vp]
+        L.inlgen_load_csr.argtypes = [C.c_char_p, C.POINTER(vp)]
+        L.inlgen_graph_from_csr.argtypes = [i64, i64, i64, vp, vp, vp, vp, C.POINTER(vp)]
+        L.inlgen_graph_values.argtypes = [vp, vp]
+        L.inlgen_powerlaw_build.argtypes = [i64, i32, i32, C.c_double, u64, i32, C.POINTER(vp)]
         L.inlgen_vector_dev.argtypes = [i64, i64, u64, i32, vp, vp]
         _lib = L
     return _lib
@@ -82,7 +88,7 @@ def rmat_tuples(scale: int, seed: int, e_begin: int, count: int):
 class HostGraph:
     """CSR on the host: row_ptr int64 [n_rows+1], col_idx int32 [nnz] (global ids)."""
 
-    def __init__(self, n_global, row_begin, row_ptr, col_idx, out_degree=None, scale=None, flags=0):
+    def __init__(self, n_global, row_begin, row_ptr, col_idx, out_degree=None, scale=None, flags=0, val=None):
         self.n_global = int(n_global)
         self.row_begin = int(row_begin)
         self.row_ptr = row_ptr
@@ -90,6 +96,7 @@ class HostGraph:
         self.out_degree = out_degree
         self.scale = scale
         self.flags = flags
+        self.val = val  # fp32 values of a loaded matrix (None for generated graphs)
 
     @property
     def n_rows(self) -> int:
@@ -122,6 +129,85 @@ def host_build(scale: int, edge_factor: int = 16, seed: int = SEED_GRAPH, flags:
     finally:
         lib().inlgen_graph_free(g)
     return HostGraph(n_global, rb, rp, ci, od, scale, flags)
+
+
+def _host_graph(g, flags=0, scale=None) -> HostGraph:
+    """Export a library host graph handle into numpy arrays (and free the handle)."""
+    try:
+        n_global, n_rows, rb, nnz, _ = _info(g)
+        rp = np.empty(n_rows + 1, dtype=np.int64)
+        ci = np.empty(max(nnz, 0), dtype=np.int32)
+        od = np.empty(n_global, dtype=np.int32) if flags & TRANSPOSE else None
+        _check(lib().inlgen_graph_export(g, _p(rp), _p(ci), _p(od) if od is not None else 0, None),
+               "inlgen_graph_export")
+        val = np.empty(max(nnz, 0), dtype=np.float32)
+        if lib().inlgen_graph_values(g, _p(val) if nnz else val.ctypes.data) != 0:
+            val = None
+    finally:
+        lib().inlgen_graph_free(g)
+    return HostGraph(n_global, rb, rp, ci, od, scale, flags, val)
+
+
+def load_mtx(path: str, flags: int = 0) -> HostGraph:
+    """MatrixMarket coordinate file -> host CSR (self-loops dropped, repeated pairs keep the first
+    value, columns sorted; SYMMETRIC adds reverses, TRANSPOSE gives the in-CSR + out_degree)."""
+    g = C.c_void_p()
+    _check(lib().inlgen_load_mtx(os.fsencode(path), flags, C.byref(g)), "inlgen_load_mtx")
+    return _host_graph(g, flags)
+
+
+def save_inlcsr(path: str, g: HostGraph) -> None:
+    """Write a host CSR (with its values / out_degree when present) as an .inlcsr file."""
+    h = C.c_void_p()
+    rp = np.ascontiguousarray(g.row_ptr, dtype=np.int64)
+    ci = np.ascontiguousarray(g.col_idx, dtype=np.int32)
+    val = None if g.val is None else np.ascontiguousarray(g.val, dtype=np.float32)
+    od = None if g.out_degree is None else np.ascontiguousarray(g.out_degree, dtype=np.int32)
+    _check(lib().inlgen_graph_from_csr(g.n_global, len(rp) - 1, g.row_begin, _p(rp), _p(ci) if ci.size else None,
+                                       _p(val) if val is not None and val.size else None,
+                                       _p(od) if od is not None and od.size else None, C.byref(h)),
+           "inlgen_graph_from_csr")
+    try:
+        _check(lib().inlgen_save_csr(os.fsencode(path), h), "inlgen_save_csr")
+    finally:
+        lib().inlgen_graph_free(h)
+
+
+def load_inlcsr(path: str) -> HostGraph:
+    g = C.c_void_p()
+    _check(lib().inlgen_load_csr(os.fsencode(path), C.byref(g)), "inlgen_load_csr")
+    # out_degree travels in the file when it was saved with one
+    n_global, n_rows, rb, nnz, _ = _info(g)
+    try:
+        rp = np.empty(n_rows + 1, dtype=np.int64)
+        ci = np.empty(max(nnz, 0), dtype=np.int32)
+        od = np.empty(max(n_global, 1), dtype=np.int32)
+        rc = lib().inlgen_graph_export(g, _p(rp), _p(ci), od.ctypes.data, None)
+        od = od[:n_global] if rc == 0 else None
+        if rc != 0:
+            _check(lib().inlgen_graph_export(g, _p(rp), _p(ci), None, None), "inlgen_graph_export")
+        val = np.empty(max(nnz, 0), dtype=np.float32)
+        if lib().inlgen_graph_values(g, val.ctypes.data) != 0:
+            val = None
+    finally:
+        lib().inlgen_graph_free(g)
+    return HostGraph(n_global, rb, rp, ci, od, None, TRANSPOSE if od is not None else 0, val)
+
+
+def powerlaw_build(n: int, dmin: int, dmax: int, mean: float, seed: int = SEED_GRAPH) -> HostGraph:
+    """Undirected configuration-model graph with a truncated power-law degree sequence."""
+    g = C.c_void_p()
+    _check(lib().inlgen_powerlaw_build(n, dmin, dmax, mean, seed, 0, C.byref(g)), "inlgen_powerlaw_build")
+    return _host_graph(g, SYMMETRIC)
+
+
+# PAPER.md P5@12491-13052: CiteSeer, 434,102 nodes, "16 million edges", degree 1..1,188, mean 73.9
+CITESEER_N, CITESEER_DMIN, CITESEER_DMAX, CITESEER_MEAN = 434102, 1, 1188, 73.9
+
+
+def citeseer_like(seed: int = SEED_GRAPH) -> HostGraph:
+    """The CiteSeer-shaped synthetic graph of SURVEY §8f NEXT-2 (symmetric CSR)."""
+    return powerlaw_build(CITESEER_N, CITESEER_DMIN, CITESEER_DMAX, CITESEER_MEAN, seed)
 
 
 def dev_build(scale: int, edge_factor: int = 16, seed: int = SEED_GRAPH, flags: int = 0,

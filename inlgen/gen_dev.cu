@@ -216,6 +216,7 @@ extern "C" void inlgen_graph_free(inlgen_graph g) {
     free(g->row_ptr);
     free(g->col_idx);
     free(g->out_degree);
+    free(g->val);
   }
   free(g);
 }

@@ -12,6 +12,7 @@ struct inlgen_graph_s {
   int64_t *row_ptr;    /* [n_rows+1] */
   int32_t *col_idx;    /* [nnz] */
   int32_t *out_degree; /* [n_global] or NULL */
+  float *val;          /* [nnz] or NULL (loaded matrices with values; host graphs only) */
 };
 
 #ifdef __cplusplus

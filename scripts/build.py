@@ -69,10 +69,10 @@ def build_oracle_par(force: bool = False) -> str:
 def build_inlgen(force: bool = False) -> str:
     out = os.path.join(ROOT, "inlgen", "libinlgen.so")
     d = os.path.join(ROOT, "inlgen")
-    srcs = [os.path.join(d, f) for f in ("gen_host.cpp", "gen_dev.cu")]
+    srcs = [os.path.join(d, f) for f in ("gen_host.cpp", "gen_dev.cu", "loader.cpp")]
     deps = srcs + glob.glob(os.path.join(d, "*.h")) + [os.path.join(ROOT, "include", "inlgen.h")]
     if force or _stale(out, deps):
-        _run([NVCC] + NVCC_COMMON + ["-shared", "-o", out] + srcs)
+        _run([NVCC] + NVCC_COMMON + ["-I", os.path.join(ROOT, "include"), "-shared", "-o", out] + srcs)
     return out
 
 
