@@ -21,8 +21,33 @@ import inlgen  # noqa: E402
 from paper_conf_icpp_liwb15_b200 import inl  # noqa: E402
 
 
+def citeseer_workload(op, torch):
+    """The CiteSeer-shaped synthetic graph (n = 434,102, ~32.1 M CSR entries, degree 1..1,188,
+    mean 73.9; inlgen.citeseer_like) on the GPU with the recipe's values / x / weights."""
+    import inlgen
+    cache = os.environ.get("INL_CITESEER_CACHE", "/tmp/inl_citeseer_seed1.inlcsr")  # regenerated if absent
+    if os.path.exists(cache):
+        h = inlgen.load_inlcsr(cache)
+    else:
+        h = inlgen.citeseer_like()
+        inlgen.save_inlcsr(cache, h)
+    rp = torch.from_numpy(h.row_ptr).cuda()
+    ci = torch.from_numpy(h.col_idx).cuda()
+    g = {"n_global": h.n_global, "row_begin": 0, "row_ptr": rp, "col_idx": ci, "out_degree": None}
+    W = {"g": g, "n": h.n_global}
+    if op == "spmv":
+        W["val"] = inlgen.values_dev(rp, ci)
+        W["x"] = inlgen.vector_dev(h.n_global)
+    else:
+        W["w"] = inlgen.weights_dev(rp, ci)
+    torch.cuda.synchronize()
+    return W
+
+
 def main():
     ap = argparse.ArgumentParser()
+    ap.add_argument("--graph", choices=["rmat", "citeseer"], default="rmat",
+                    help="citeseer: the CiteSeer-shaped graph of PAPER.md P5@12491 (inlgen.citeseer_like)")
     ap.add_argument("--scale", type=int, default=23)
     ap.add_argument("--sources", type=int, default=3)
     ap.add_argument("--only", type=str, default="", help="NAME[:LBT] — run one variant (for ncu)")
@@ -31,7 +56,7 @@ def main():
     stream = torch.cuda.Stream(0)
     torch.cuda.set_stream(stream)
     ctx = inl.Ctx(0)
-    W = bench.build_workload("sssp", a.scale, 16, 1, 0, torch)
+    W = citeseer_workload("sssp", torch) if a.graph == "citeseer" else bench.build_workload("sssp", a.scale, 16, 1, 0, torch)
     g = W["g"]
     A = inl.Csr(g["row_ptr"], g["col_idx"], g["n_global"])
     srcs = inlgen.sources(g["row_ptr"].cpu().numpy(), a.sources)[: a.sources]
@@ -66,7 +91,7 @@ def main():
             t1 = ms
         print(json.dumps({"template": name, "lbTHRES": lbt, "bins": kw, "ms_per_source": round(ms, 4),
                           "speedup_vs_T1": round(t1 / ms, 2), "relaxations": relax // len(srcs),
-                          "scale": a.scale, "sources": srcs}), flush=True)
+                          "scale": a.scale, "graph": a.graph, "sources": srcs}), flush=True)
         del plan
 
 
