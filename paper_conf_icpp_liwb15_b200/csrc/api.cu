@@ -318,6 +318,59 @@ void comm_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, nc
   INL_NCCL(ncclAllReduce(buf, buf, (size_t)count, dt, op, ctx->comm, st));
 }
 
+void comm_barrier(inl_ctx ctx, cudaStream_t st) {
+  if (!st) st = ctx->stream;
+  if (ctx->loop) return loop_barrier(ctx, st);
+  INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
+  // a one-word allreduce: every rank's prior work on `st` precedes it, every rank's later work
+  // follows its completion (NCCL's kernels order the peers' streams)
+  int32_t *w = (int32_t *)ctx->s_bar.get(16);
+  INL_NCCL(ncclAllReduce(w, w, 1, ncclInt32, ncclMax, ctx->comm, st));
+}
+
+static void close_peer_maps(inl_ctx ctx) {
+  for (void *p : ctx->ipc_open)
+    if (p) cudaIpcCloseMemHandle(p);
+  ctx->ipc_open.clear();
+  ctx->peer_bases.clear();
+  ctx->peer_mine = nullptr;
+  ctx->peer_bytes = 0;
+}
+
+const std::vector<void *> &comm_peer_bases(inl_ctx ctx, void *mine, size_t bytes) {
+  if (ctx->peer_mine == mine && ctx->peer_bytes == bytes && !ctx->peer_bases.empty()) return ctx->peer_bases;
+  close_peer_maps(ctx);
+  if (ctx->loop) {
+    loop_exchange_ptrs(ctx, mine, ctx->peer_bases);
+  } else {
+    INL_CHECK(ctx->comm != nullptr, "NCCL communicator not initialised (inl_comm_init)");
+    const int P = ctx->nranks;
+    cudaIpcMemHandle_t h;
+    INL_CUDA(cudaIpcGetMemHandle(&h, mine));
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+    char *dh = (char *)ctx->s_tmp.get(64 * (size_t)(P + 1));
+    INL_CUDA(cudaMemcpyAsync(dh + 64 * (size_t)ctx->rank, &h, 64, cudaMemcpyHostToDevice, ctx->stream));
+    INL_NCCL(ncclAllGather(dh + 64 * (size_t)ctx->rank, dh, 64, ncclUint8, ctx->comm, ctx->stream));
+    std::vector<cudaIpcMemHandle_t> all(P);
+    INL_CUDA(cudaMemcpyAsync(all.data(), dh, 64 * (size_t)P, cudaMemcpyDeviceToHost, ctx->stream));
+    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx->peer_bases.assign(P, nullptr);
+    for (int q = 0; q < P; ++q) {
+      if (q == ctx->rank) {
+        ctx->peer_bases[q] = mine;
+        continue;
+      }
+      void *p = nullptr;
+      INL_CUDA(cudaIpcOpenMemHandle(&p, all[q], cudaIpcMemLazyEnablePeerAccess));
+      ctx->ipc_open.push_back(p);
+      ctx->peer_bases[q] = p;
+    }
+  }
+  ctx->peer_mine = mine;
+  ctx->peer_bytes = bytes;
+  return ctx->peer_bases;
+}
+
 cudaStream_t comm_stream(inl_ctx ctx) {
   if (!ctx->comm_stream) INL_CUDA(cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking));
   return ctx->comm_stream;
@@ -387,6 +440,7 @@ static void free_ctx(inl_ctx ctx) {
   cudaGetDevice(&old);
   cudaSetDevice(ctx->device);
   cudaStreamSynchronize(ctx->stream);
+  close_peer_maps(ctx);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   if (ctx->loop) loop_release(ctx->loop);
   if (ctx->comm_stream) {

@@ -88,6 +88,7 @@ struct SsspOp {
   __device__ __forceinline__ uint32_t load(int32_t u) const {
     return *(volatile uint32_t *)(dist + row_begin + u);
   }
+  __device__ __forceinline__ void fence() const {}
   __device__ __forceinline__ void improve(int32_t v, uint32_t nd, int32_t *q, int *cnt) const {
     const uint32_t old = atomicMin(dist + v, nd);
     if (nd < old) {
@@ -155,9 +156,22 @@ struct BfsOp {
   uint64_t pol_stream;
   const int64_t *rp = nullptr;       // !DIST: degree sum of the next frontier -> *mf
   unsigned long long *mf = nullptr;  //   (Beamer's m_f, for the direction switch)
+  // NEXT-1 fused exchange (DIST): a discovered vertex v sets its bit in the next-frontier
+  // bitmap of its OWNER q = v / B, in q's memory (NVLink peer memory; the same device for the
+  // loopback), during the expansion itself — no byte map, no allreduce
+  uint32_t *const *xtab = nullptr;   // [P] owners' bitmaps of this level
+  int64_t B = 0;                     // row block
+  __device__ __forceinline__ void xset(int32_t v) const {
+    atomicOr(xtab[v / B] + (v >> 5), 1u << (v & 31));
+  }
+  __device__ __forceinline__ void fence() const {
+    if (xtab) __threadfence_system();  // the peers read these bits after the barrier
+  }
   __device__ __forceinline__ uint32_t load(int32_t) const { return 0u; }
   __device__ __forceinline__ void visit(int32_t v, int32_t *q, int *cnt) const {
-    if (enqueue) {
+    if (!enqueue && xtab) {
+      xset(v);
+    } else if (enqueue) {
       const uint32_t bit = 1u << (v & 31);
       const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
       if (!(old & bit)) {
@@ -186,6 +200,12 @@ struct BfsOp {
     for (int j = 0; j < K; ++j)
       if (!((bw[j] >> (vv[j] & 31)) & 1u)) cand |= 1u << j;
     if (!enqueue) {
+      if (xtab) {
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+          if ((cand >> j) & 1u) xset(vv[j]);
+        return;
+      }
 #pragma unroll
       for (int j = 0; j < K; ++j)
         if ((cand >> j) & 1u) next[vv[j]] = 1;
@@ -360,6 +380,7 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
     for (int q = 0; q < NW; ++q) s += red[q];
     if (s) atomicAdd(a.relaxed, s);
   }
+  op.fence();
 }
 
 // Default expansion (dbuf-shared, P5@3623, B200 form): every frontier vertex of the
@@ -476,6 +497,7 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
     for (int q = 0; q < NW; ++q) s += red[q];
     if (s) atomicAdd(a.relaxed, s);
   }
+  op.fence();
 }
 
 // Grid bin (dbuf-global, P5@2721): pieces of grid_chunk edges of the large-degree
@@ -511,6 +533,7 @@ __global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
       op.edges(du, kk, vv, in, a.Fout, a.fcount);
     }
   }
+  op.fence();
 }
 
 __global__ void k_init_sssp(uint32_t *dist, int64_t n, int64_t s) {
@@ -635,6 +658,41 @@ __global__ void k_bfs_apply(const uint8_t *__restrict__ next, int64_t n, int32_t
       atomicOr(bm + (v >> 5), 1u << (v & 31));
       if (v >= row_begin && v < row_begin + n_rows) push(q, cnt, (int32_t)(v - row_begin));
     }
+  }
+}
+
+// NEXT-1 apply (P > 1): the level's new-frontier bitmap is the OR over the owners' buffers (an
+// owner's buffer holds the bits every rank set for its vertices; a word straddling two row
+// blocks reads both).  New vertices (not yet visited) get level L+1 on EVERY rank — the level
+// vector stays replicated with no allgather — and the owned ones form the next local frontier.
+// *total counts the new vertices of the whole graph: the same on every rank, so the ranks agree
+// on termination without a collective.
+__global__ void k_bfs_apply_xbits(uint32_t *const *__restrict__ xtab, int64_t B, int64_t n, uint32_t *bm,
+                                  int32_t *level, int L, int64_t row_begin, int64_t n_rows, int32_t *q, int *cnt,
+                                  unsigned long long *total) {
+  const int64_t nwords = (n + 31) / 32;
+  const int64_t nn = (nwords + 31) / 32 * 32;
+  unsigned long long c = 0;
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nn; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t nw = 0;
+    if (w < nwords) {
+      const int64_t lo = w * 32, hi = min(lo + 32, n);
+      uint32_t bits = 0;
+      for (int64_t o = lo / B; o <= (hi - 1) / B; ++o) bits |= __ldcg(xtab[o] + w);
+      nw = bits & ~bm[w];
+      if (nw) {
+        bm[w] |= nw;
+        c += (unsigned long long)__popc(nw);
+        for (uint32_t b = nw; b; b &= b - 1) {
+          const int64_t v = lo + __ffs(b) - 1;
+          level[v] = L + 1;
+          if (v >= row_begin && v < row_begin + n_rows) push(q, cnt, (int32_t)(v - row_begin));
+        }
+      }
+    }
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(total, c);
+    c = 0;
   }
 }
 
@@ -1375,9 +1433,35 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
   uint32_t *bm = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * ((n + 31) / 32 + 1));
-  uint8_t *next = DIST ? (uint8_t *)ctx->s_e.get(n + 1) : nullptr;
+  // P > 1 exchange: NEXT-1 bit-packed owner bitmaps (default) or the r01 byte map + allreduce-max
+  // (INL_BFS_EXCHANGE=bytemap, measurement switch)
+  const char *xe = getenv("INL_BFS_EXCHANGE");
+  const bool xbits = DIST && !(xe && std::string(xe) == "bytemap");
+  uint8_t *next = DIST && !xbits ? (uint8_t *)ctx->s_e.get(n + 1) : nullptr;
   k_init_bfs<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(level, bm, n, source);
   INL_CUDA(cudaGetLastError());
+  const int P = DIST ? ctx->nranks : 1;
+  const int64_t B = (n + P - 1) / P;
+  const int64_t xw = ((n + 31) / 32 + 31) / 32 * 32;  // words per level buffer (128-B aligned)
+  uint32_t *xb = nullptr;
+  uint32_t **xtab = nullptr;
+  unsigned long long *xtotal = (unsigned long long *)(f.counts + 10);
+  if (xbits && n > 0) {
+    // three level buffers (level L writes buffer L % 3; a rank clears buffer (L+1) % 3 before
+    // its level-L expansion: every rank read it at level L-2, before the level L-1 barrier, and
+    // peers write it only after the level-L barrier) — one barrier per level
+    const size_t bytes = sizeof(uint32_t) * 3 * (size_t)xw;
+    xb = (uint32_t *)ctx->s_xch.get(bytes);
+    INL_CUDA(cudaMemsetAsync(xb, 0, bytes, st));
+    const std::vector<void *> &bases = comm_peer_bases(ctx, ctx->s_xch.p, ctx->s_xch.bytes);
+    std::vector<uint32_t *> tab((size_t)3 * P);
+    for (int bb = 0; bb < 3; ++bb)
+      for (int q = 0; q < P; ++q) tab[(size_t)bb * P + q] = (uint32_t *)bases[q] + (size_t)bb * xw;
+    xtab = (uint32_t **)ctx->s_xtab.get(sizeof(uint32_t *) * tab.size());
+    INL_CUDA(cudaMemcpyAsync(xtab, tab.data(), sizeof(uint32_t *) * tab.size(), cudaMemcpyHostToDevice, st));
+    INL_CUDA(cudaStreamSynchronize(st));  // `tab` is a host temporary
+    comm_barrier(ctx);  // every rank's buffers are zero before any peer writes into them
+  }
   int nF = 0;
   if (source >= G.row_begin && source < G.row_begin + G.n_rows) {
     const int32_t s_local = (int32_t)(source - G.row_begin);
@@ -1519,6 +1603,26 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
         queue_ok = true;
       }
       bu = want_bu;
+      ++L;
+    } else if (xbits) {  // NEXT-1: bits straight into the owners' buffers, one barrier per level
+      const int buf = L % 3;
+      INL_CUDA(cudaMemsetAsync(xb + (size_t)((L + 1) % 3) * xw, 0, sizeof(uint32_t) * xw, st));
+      BfsOp op{bm, level, nullptr, n, L, false, 0};
+      op.xtab = xtab + (size_t)buf * P;
+      op.B = B;
+      expand(ctx, G, b, f, nF, op);
+      comm_barrier(ctx);
+      INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+      INL_CUDA(cudaMemsetAsync(xtotal, 0, sizeof(unsigned long long), st));
+      k_bfs_apply_xbits<<<grid_for((n + 31) / 32, ctx->num_sms), 256, 0, st>>>(xtab + (size_t)buf * P, B, n, bm, level,
+                                                                                L, G.row_begin, G.n_rows, f.F, f.counts,
+                                                                                xtotal);
+      INL_CUDA(cudaGetLastError());
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 48, cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaStreamSynchronize(st));
+      nF = ((volatile int *)ctx->pinned)[0];
+      const unsigned long long tot = *(volatile unsigned long long *)((int *)ctx->pinned + 10);
+      if (tot == 0) break;
       ++L;
     } else {
       INL_CUDA(cudaMemsetAsync(next, 0, n + 1, st));

@@ -138,6 +138,14 @@ struct inl_ctx_s {
   cudaStream_t comm_stream = nullptr;  // second stream: exchanges overlapped with the gather
   cudaEvent_t events[inl::kCtxEvents] = {};
   void *sssp_graph = nullptr;  // cached executable graph of the one-GPU SSSP loop (frontier.cu)
+  // peer mappings of one exchange buffer (comm_peer_bases): every rank's base pointer, the
+  // local buffer they belong to, and the CUDA IPC mappings to close when it changes
+  std::vector<void *> peer_bases, ipc_open;
+  void *peer_mine = nullptr;
+  size_t peer_bytes = 0;
+  inl::DevBuf s_xch;   // NEXT-1 exchange buffers (frontier bitmaps peers write into)
+  inl::DevBuf s_xtab;  // device tables of peer pointers into s_xch
+  inl::DevBuf s_bar;   // NCCL barrier word
   int nranks = 1, rank = 0;
   // scratch
   inl::DevBuf s_tmp, s_a, s_b, s_c, s_d, s_e, s_f, s_g;

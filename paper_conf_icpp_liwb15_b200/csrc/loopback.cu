@@ -186,6 +186,19 @@ void loop_allreduce(inl_ctx ctx, void *buf, int64_t count, ncclDataType_t dt, nc
   if (count > 0) INL_CUDA(cudaMemcpyAsync(buf, tmp, es * (size_t)count, cudaMemcpyDeviceToDevice, st));
 }
 
+void loop_barrier(inl_ctx ctx, cudaStream_t st) {
+  phase_in(ctx, ctx->loop, nullptr, nullptr, nullptr, st);
+  phase_out(ctx, ctx->loop, st);
+}
+
+void loop_exchange_ptrs(inl_ctx ctx, void *mine, std::vector<void *> &out) {
+  LoopGroup *g = ctx->loop;
+  phase_in(ctx, g, mine, mine, nullptr, ctx->stream);
+  out.assign(g->nranks, nullptr);
+  for (int q = 0; q < g->nranks; ++q) out[q] = g->dst[q];
+  phase_out(ctx, g, ctx->stream);
+}
+
 void loop_abort(inl_ctx ctx) {
   if (ctx && ctx->loop) ctx->loop->abort();
 }
