@@ -85,11 +85,33 @@ struct SsspOp {
   int32_t *far;         // far pile (each vertex at most once: `infar` bitmap)
   int *far_count;
   uint32_t *infar;
+  // NEXT-1 sparse exchange (DIST): vertex v's distance is OWNED by rank q = v / B; a
+  // relaxation that beats this rank's (stale, upper-bound) copy dist[v] does atomicMin in the
+  // owner's array (peer memory) and, if that improved it, sets v's bit in the owner's
+  // changed-bitmap of the round; nimp counts those improvements (summed by the one allreduce
+  // per round, which is also the barrier and the termination test)
+  uint32_t *const *xd = nullptr;   // [P] owners' distance arrays (xd[rank] == dist)
+  uint32_t *const *xc = nullptr;   // [P] owners' changed bitmaps of this round
+  int64_t B = 0;
+  unsigned int *nimp = nullptr;
+  __device__ __forceinline__ bool xrelax(int32_t v, uint32_t nd) const {
+    uint32_t *o = xd[v / B];
+    if (o != dist) atomicMin(dist + v, nd);  // keep the local filter tight
+    if (atomicMin(o + v, nd) <= nd) return false;
+    atomicOr(xc[v / B] + (v >> 5), 1u << (v & 31));
+    return true;
+  }
   __device__ __forceinline__ uint32_t load(int32_t u) const {
     return *(volatile uint32_t *)(dist + row_begin + u);
   }
-  __device__ __forceinline__ void fence() const {}
+  __device__ __forceinline__ void fence() const {
+    if (xd) __threadfence_system();  // the owners read these after the round's allreduce
+  }
   __device__ __forceinline__ void improve(int32_t v, uint32_t nd, int32_t *q, int *cnt) const {
+    if (xd) {
+      if (xrelax(v, nd)) atomicAdd(nimp, 1u);
+      return;
+    }
     const uint32_t old = atomicMin(dist + v, nd);
     if (nd < old) {
       if (enqueue) {
@@ -120,6 +142,15 @@ struct SsspOp {
     for (int j = 0; j < K; ++j) nd[j] = in[j] ? du[j] + ld_stream_pol(w + kk[j], pol_stream) : 0xFFFFFFFFu;
 #pragma unroll
     for (int j = 0; j < K; ++j) dv[j] = in[j] ? dist[vv[j]] : 0u;
+    if (xd) {  // NEXT-1: improvements go to the owners
+      unsigned c = 0;
+#pragma unroll
+      for (int j = 0; j < K; ++j)
+        if (nd[j] < dv[j] && xrelax(vv[j], nd[j])) ++c;
+      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+      if ((threadIdx.x & 31) == 0 && c) atomicAdd(nimp, c);
+      return;
+    }
 #pragma unroll
     for (int j = 0; j < K; ++j) old[j] = nd[j] < dv[j] ? atomicMin(dist + vv[j], nd[j]) : 0u;
     unsigned imp = 0u;
@@ -636,6 +667,19 @@ __global__ void k_sssp_collect(const uint32_t *__restrict__ dist, uint32_t *__re
     if (d < prev[v]) {
       prev[v] = d;
       push(q, cnt, (int32_t)v);
+    }
+  }
+}
+
+// NEXT-1: the owned vertices whose distance improved this round (their bits in this rank's
+// changed-bitmap, set by every rank's relaxations) -> next local frontier
+__global__ void k_sssp_collect_xbits(const uint32_t *__restrict__ chg, int64_t row_begin, int64_t n_rows, int32_t *q,
+                                     int *cnt) {
+  const int64_t w0 = row_begin / 32, w1 = (row_begin + n_rows + 31) / 32;
+  for (int64_t w = w0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < w1; w += (int64_t)gridDim.x * blockDim.x) {
+    for (uint32_t b = chg[w]; b; b &= b - 1) {
+      const int64_t v = w * 32 + __ffs(b) - 1;
+      if (v >= row_begin && v < row_begin + n_rows) push(q, cnt, (int32_t)(v - row_begin));
     }
   }
 }
@@ -1341,7 +1385,32 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   int *farcnt = nullptr;
   int nfar = 0;
   uint32_t delta = 0xFFFFFFFFu, thr = 0xFFFFFFFFu;
-  if (DIST) {
+  // P > 1 exchange: NEXT-1 sparse owner updates (default) or the r01 dense allreduce-min of the
+  // whole distance vector (INL_SSSP_EXCHANGE=dense, measurement switch)
+  const char *xe = getenv("INL_SSSP_EXCHANGE");
+  const bool xsparse = DIST && n > 0 && !(xe && std::string(xe) == "dense");
+  const int P = DIST ? ctx->nranks : 1;
+  const int64_t Bk = (n + P - 1) / P;
+  const int64_t xw = ((n + 31) / 32 + 31) / 32 * 32;  // words per changed-bitmap (128-B aligned)
+  const int64_t dlen = (Bk * P + 31) / 32 * 32;      // padded replicated distance vector
+  uint32_t *xchg = nullptr, **xtab = nullptr;
+  unsigned int *nimp = (unsigned int *)(f.counts + 3);
+  if (xsparse) {
+    // one exchange buffer: [distances (dlen)] [3 changed-bitmaps (xw each), round r uses r % 3]
+    const size_t bytes = sizeof(uint32_t) * ((size_t)dlen + 3 * (size_t)xw);
+    D = (uint32_t *)ctx->s_xch.get(bytes);
+    xchg = D + dlen;
+    INL_CUDA(cudaMemsetAsync(xchg, 0, sizeof(uint32_t) * 3 * (size_t)xw, st));
+    const std::vector<void *> &bases = comm_peer_bases(ctx, ctx->s_xch.p, ctx->s_xch.bytes);
+    std::vector<uint32_t *> tab((size_t)4 * P);  // [0]: distances, [1 + r]: changed-bitmap r
+    for (int q = 0; q < P; ++q) {
+      tab[q] = (uint32_t *)bases[q];
+      for (int r = 0; r < 3; ++r) tab[(size_t)(1 + r) * P + q] = (uint32_t *)bases[q] + dlen + (size_t)r * xw;
+    }
+    xtab = (uint32_t **)ctx->s_xtab.get(sizeof(uint32_t *) * tab.size());
+    INL_CUDA(cudaMemcpyAsync(xtab, tab.data(), sizeof(uint32_t *) * tab.size(), cudaMemcpyHostToDevice, st));
+    INL_CUDA(cudaStreamSynchronize(st));
+  } else if (DIST) {
     D = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * (n + 1));
     prev = (uint32_t *)ctx->s_e.get(sizeof(uint32_t) * (G.n_rows + 1));
   } else {
@@ -1366,7 +1435,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
     INL_CUDA(cudaMemcpyAsync(f.F, &s_local, sizeof(int32_t), cudaMemcpyHostToDevice, st));
     nF = 1;
   }
-  if (DIST) k_copy_u32<<<grid_for(G.n_rows, ctx->num_sms), 256, 0, st>>>(D + G.row_begin, prev, G.n_rows);
+  if (DIST && !xsparse) k_copy_u32<<<grid_for(G.n_rows, ctx->num_sms), 256, 0, st>>>(D + G.row_begin, prev, G.n_rows);
+  if (xsparse) comm_barrier(ctx);  // every rank's distances / bitmaps are initialised before peers write
   int iters = 0;
   int64_t ftotal = 0;
   for (;;) {
@@ -1402,6 +1472,26 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       nF = ((volatile int *)ctx->pinned)[0];
       nfar = ((volatile int *)ctx->pinned)[1];
       std::swap(f.F, f.Fout);
+    } else if (xsparse) {
+      const int r = iters % 3;
+      INL_CUDA(cudaMemsetAsync(xchg + (size_t)((iters + 1) % 3) * xw, 0, sizeof(uint32_t) * xw, st));
+      INL_CUDA(cudaMemsetAsync(nimp, 0, sizeof(unsigned int), st));
+      SsspOp op{D, w, nullptr, nullptr, iters, G.row_begin, false, 0, 0xFFFFFFFFu, nullptr, nullptr, nullptr};
+      op.xd = xtab;
+      op.xc = xtab + (size_t)(1 + r) * P;
+      op.B = Bk;
+      op.nimp = nimp;
+      expand(ctx, G, b, f, nF, op);
+      comm_allreduce(ctx, nimp, 1, ncclUint32, ncclSum);  // the round's barrier + termination test
+      ++iters;
+      INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
+      k_sssp_collect_xbits<<<grid_for((G.n_rows + 31) / 32 + 1, ctx->num_sms), 256, 0, st>>>(
+          xchg + (size_t)r * xw, G.row_begin, G.n_rows, f.F, f.counts);
+      INL_CUDA(cudaGetLastError());
+      INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 16, cudaMemcpyDeviceToHost, st));
+      INL_CUDA(cudaStreamSynchronize(st));
+      nF = ((volatile int *)ctx->pinned)[0];
+      if (((volatile unsigned int *)ctx->pinned)[3] == 0u) break;
     } else {
       // flag word D[n] = 1 ("no change"), cleared by any improvement on any rank
       const uint32_t one = 1u;
@@ -1420,6 +1510,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       nF = read_count(ctx, f.counts);
     }
   }
+  if (xsparse)  // replicate: the owners' slices (in place, padded to P equal blocks)
+    comm_allgather(ctx, D + (size_t)ctx->rank * Bk, D, Bk, ncclUint32, nullptr, nullptr);
   if (DIST)
     INL_CUDA(cudaMemcpyAsync(dist, D, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, st));
   finish_stats(ctx, f, stats, iters, ftotal);

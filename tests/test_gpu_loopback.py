@@ -189,7 +189,14 @@ def _frontier_ranks(P, g, w, sources, use_plan=True):
 
 
 @pytest.mark.parametrize("P", PS)
-def test_sssp_bfs_cfg1_bit_exact(g12_sym, P):
+@pytest.mark.parametrize("exchange", ["fused", "collective"])
+def test_sssp_bfs_cfg1_bit_exact(g12_sym, P, exchange, monkeypatch):
+    """exchange = fused: NEXT-1 (BFS bits set in the owners' bitmaps, SSSP improvements
+    sent to the owners, peer memory; the default); collective: the r01 byte-map allreduce-max /
+    dense allreduce-min over the whole vector."""
+    if exchange == "collective":
+        monkeypatch.setenv("INL_BFS_EXCHANGE", "bytemap")
+        monkeypatch.setenv("INL_SSSP_EXCHANGE", "dense")
     g, w = g12_sym
     srcs = inlgen.sources(g.row_ptr, 8)
     res = _frontier_ranks(P, g, w, srcs)
