@@ -5,8 +5,13 @@
 #include <cstdarg>
 #include <cstdio>
 #include <algorithm>
+#include <chrono>
+#include <cstdlib>
 #include <cstring>
+#include <thread>
 #include <new>
+
+#include <nvtx3/nvToolsExt.h>
 
 #include "comm.h"
 #include "inl_internal.cuh"
@@ -16,6 +21,38 @@
 namespace inl {
 
 void raise(inl_status code, const std::string &msg) { throw Error{code, msg}; }
+
+NvtxRange::NvtxRange(const char *name) { nvtxRangePushA(name); }
+NvtxRange::~NvtxRange() { nvtxRangePop(); }
+
+void ctx_sync(inl_ctx ctx) {
+  if (!ctx->comm) {
+    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    return;
+  }
+  static double limit_s = -1.0;
+  if (limit_s < 0) {
+    const char *e = getenv("INL_NCCL_TIMEOUT_S");
+    limit_s = e ? atof(e) : 600.0;
+  }
+  const auto t0 = std::chrono::steady_clock::now();
+  for (long spin = 0;; ++spin) {
+    const cudaError_t q = cudaStreamQuery(ctx->stream);
+    if (q == cudaSuccess) return;
+    if (q != cudaErrorNotReady) INL_CUDA(q);
+    ncclResult_t r = ncclSuccess;
+    const ncclResult_t qr = ncclCommGetAsyncError(ctx->comm, &r);
+    const bool failed = qr != ncclSuccess || (r != ncclSuccess && r != ncclInProgress);
+    const double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (failed || dt > limit_s) {
+      ncclCommAbort(ctx->comm);
+      ctx->comm = nullptr;
+      raise(INL_ERR_NCCL, failed ? std::string("NCCL asynchronous error: ") + ncclGetErrorString(r)
+                                 : "NCCL collective did not complete within INL_NCCL_TIMEOUT_S; communicator aborted");
+    }
+    if (spin > 2000) std::this_thread::sleep_for(std::chrono::microseconds(20));
+  }
+}
 
 void *DevBuf::get(size_t need) {
   if (need == 0) need = 16;
@@ -537,6 +574,7 @@ inl_status inl_comm_init_loopback(inl_ctx ctx, inl_loop group, int32_t rank) {
 }
 
 inl_status inl_plan_create(inl_ctx ctx, const inl_csr *A, const inl_bins *bins, inl_plan *out) {
+  NvtxRange nvtx_("inl_plan_create");
   if (!ctx || ctx->closed) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL or destroyed");
   inl_plan p = nullptr;
   inl_status s = guarded(ctx, [&] {
@@ -586,6 +624,7 @@ inl_status inl_plan_destroy(inl_plan plan) {
 }
 
 inl_status inl_csr_validate(inl_ctx ctx, const inl_csr *A) {
+  NvtxRange nvtx_("inl_csr_validate");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(A);
@@ -597,6 +636,7 @@ inl_status inl_csr_validate(inl_ctx ctx, const inl_csr *A) {
 
 inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y,
                     inl_plan plan) {
+  NvtxRange nvtx_("inl_spmv");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(A);
@@ -615,6 +655,7 @@ inl_status inl_spmv(inl_ctx ctx, const inl_csr *A, const float *val, const float
 
 inl_status inl_spmv_allgather(inl_ctx ctx, const inl_csr *A, const float *val, const float *x, float *y_global,
                               inl_plan plan) {
+  NvtxRange nvtx_("inl_spmv_allgather");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(A);
@@ -643,6 +684,7 @@ inl_status inl_spmv_allgather(inl_ctx ctx, const inl_csr *A, const float *val, c
 
 inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_degree, float damping,
                         int32_t iterations, float *rank, inl_plan plan) {
+  NvtxRange nvtx_("inl_pagerank");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(A_in);
@@ -669,6 +711,7 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
 
 inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source, uint32_t *dist,
                     inl_stats *stats, inl_plan plan) {
+  NvtxRange nvtx_("inl_sssp");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(G);
@@ -685,12 +728,13 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
     sssp_run(ctx, d, b, dw, source, o.dev, stats);
     finish_out(ctx, o);
-    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx_sync(ctx);
   });
 }
 
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level, inl_stats *stats,
                    inl_plan plan) {
+  NvtxRange nvtx_("inl_bfs");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(G);
@@ -705,12 +749,13 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
     bfs_run(ctx, d, b, source, o.dev, stats, plan && plan->symmetric);
     finish_out(ctx, o);
-    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx_sync(ctx);
   });
 }
 
 inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t n_sources, double *bc,
                   inl_stats *stats, inl_plan plan) {
+  NvtxRange nvtx_("inl_bc");
   if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
   return guarded(ctx, [&] {
     check_csr(G);
@@ -726,7 +771,7 @@ inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t
     StagedOut<double> o = stage_out(ctx->h_y, bc, G->n_global);
     bc_run(ctx, d, sources, n_sources, o.dev, stats, plan && plan->symmetric);
     finish_out(ctx, o);
-    INL_CUDA(cudaStreamSynchronize(ctx->stream));
+    ctx_sync(ctx);
   });
 }
 

@@ -1082,7 +1082,7 @@ FrontierBufs frontier_bufs(inl_ctx ctx, const inl_csr &G, const Bins &b) {
 void check_overflow(inl_ctx ctx, const FrontierBufs &f) {
   int h = 0;
   INL_CUDA(cudaMemcpyAsync(&h, f.counts + 2, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
-  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  ctx_sync(ctx);
   if (h) raise(INL_ERR_INTERNAL, "frontier grid buffer overflow (capacity " + std::to_string(f.gcap) + " pieces)");
 }
 
@@ -1111,7 +1111,7 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
 
 int read_count(inl_ctx ctx, const int *d) {
   INL_CUDA(cudaMemcpyAsync(ctx->pinned, d, sizeof(int), cudaMemcpyDeviceToHost, ctx->stream));
-  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  ctx_sync(ctx);
   return *(volatile int *)ctx->pinned;
 }
 
@@ -1120,7 +1120,7 @@ void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_
   if (!st) return;
   unsigned long long r = 0;
   INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, ctx->stream));
-  INL_CUDA(cudaStreamSynchronize(ctx->stream));
+  ctx_sync(ctx);
   st->iterations = iters;
   st->edges_relaxed = (int64_t)r;
   st->frontier_total = ftotal;
@@ -1195,7 +1195,7 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
     }
     INL_CUDA(cudaGetLastError());
     INL_CUDA(cudaMemcpyAsync(hs, dy.s, sizeof(SsspDev), cudaMemcpyDeviceToHost, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
     ++syncs;
     if (((volatile SsspDev *)hs)->done) break;
     if (batch < 16) batch *= 2;
@@ -1204,7 +1204,7 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   if (stats) {
     unsigned long long r = 0;
     INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
     stats->iterations = hs->iter;
     stats->edges_relaxed = (int64_t)r;
     stats->frontier_total = (int64_t)hs->ftotal;
@@ -1340,14 +1340,14 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   }
   SsspDev *hs = (SsspDev *)ctx->pinned;
   INL_CUDA(cudaMemcpyAsync(hs, dy.s, sizeof(SsspDev), cudaMemcpyDeviceToHost, st));
-  INL_CUDA(cudaStreamSynchronize(st));
+  ctx_sync(ctx);
   if (((volatile SsspDev *)hs)->done == 2)
     raise(INL_ERR_INTERNAL, "sssp graph loop exceeded its step bound");
   check_overflow(ctx, f);
   if (stats) {
     unsigned long long r = 0;
     INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
     stats->iterations = hs->iter;
     stats->edges_relaxed = (int64_t)r;
     stats->frontier_total = (int64_t)hs->ftotal;
@@ -1409,7 +1409,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
     }
     xtab = (uint32_t **)ctx->s_xtab.get(sizeof(uint32_t *) * tab.size());
     INL_CUDA(cudaMemcpyAsync(xtab, tab.data(), sizeof(uint32_t *) * tab.size(), cudaMemcpyHostToDevice, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
   } else if (DIST) {
     D = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * (n + 1));
     prev = (uint32_t *)ctx->s_e.get(sizeof(uint32_t) * (G.n_rows + 1));
@@ -1455,7 +1455,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
         INL_CUDA(cudaGetLastError());
         INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, sizeof(int), cudaMemcpyDeviceToHost, st));
         INL_CUDA(cudaMemcpyAsync((int *)ctx->pinned + 1, farcnt + 1, sizeof(int), cudaMemcpyDeviceToHost, st));
-        INL_CUDA(cudaStreamSynchronize(st));
+        ctx_sync(ctx);
         nF = ((volatile int *)ctx->pinned)[0];
         nfar = ((volatile int *)ctx->pinned)[1];
         std::swap(far_a, far_b);
@@ -1468,7 +1468,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       ++iters;
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, sizeof(int), cudaMemcpyDeviceToHost, st));
       INL_CUDA(cudaMemcpyAsync((int *)ctx->pinned + 1, farcnt, sizeof(int), cudaMemcpyDeviceToHost, st));
-      INL_CUDA(cudaStreamSynchronize(st));
+      ctx_sync(ctx);
       nF = ((volatile int *)ctx->pinned)[0];
       nfar = ((volatile int *)ctx->pinned)[1];
       std::swap(f.F, f.Fout);
@@ -1489,7 +1489,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
           xchg + (size_t)r * xw, G.row_begin, G.n_rows, f.F, f.counts);
       INL_CUDA(cudaGetLastError());
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 16, cudaMemcpyDeviceToHost, st));
-      INL_CUDA(cudaStreamSynchronize(st));
+      ctx_sync(ctx);
       nF = ((volatile int *)ctx->pinned)[0];
       if (((volatile unsigned int *)ctx->pinned)[3] == 0u) break;
     } else {
@@ -1501,7 +1501,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       comm_allreduce(ctx, D, n + 1, ncclUint32, ncclMin);
       ++iters;
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, D + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
-      INL_CUDA(cudaStreamSynchronize(st));
+      ctx_sync(ctx);
       if (*(volatile uint32_t *)ctx->pinned == 1u) break;
       INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
       k_sssp_collect<<<grid_for(G.n_rows, ctx->num_sms), 256, 0, st>>>(D, prev, G.row_begin, G.n_rows,
@@ -1551,7 +1551,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       for (int q = 0; q < P; ++q) tab[(size_t)bb * P + q] = (uint32_t *)bases[q] + (size_t)bb * xw;
     xtab = (uint32_t **)ctx->s_xtab.get(sizeof(uint32_t *) * tab.size());
     INL_CUDA(cudaMemcpyAsync(xtab, tab.data(), sizeof(uint32_t *) * tab.size(), cudaMemcpyHostToDevice, st));
-    INL_CUDA(cudaStreamSynchronize(st));  // `tab` is a host temporary
+    ctx_sync(ctx);  // `tab` is a host temporary
     comm_barrier(ctx);  // every rank's buffers are zero before any peer writes into them
   }
   int nF = 0;
@@ -1577,7 +1577,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   double m_u = (double)G.nnz;
   auto read_level = [&](int *nf, unsigned long long *mfn) {
     INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 48, cudaMemcpyDeviceToHost, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
     *nf = ((volatile int *)ctx->pinned)[0];
     *mfn = *(volatile unsigned long long *)((int *)ctx->pinned + 10);
     m_u -= (double)*mfn;
@@ -1633,7 +1633,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
             INL_CUDA(cub::DevicePartition::If(ctx->s_tmp.get(need), need, iota, bl_s[0], bl_l[0], none, f.counts + 4,
                                               (int)n, sm, lg, st));
             INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts + 4, 2 * sizeof(int), cudaMemcpyDeviceToHost, st));
-            INL_CUDA(cudaStreamSynchronize(st));
+            ctx_sync(ctx);
             n_small = ((volatile int *)ctx->pinned)[0];
             n_large = ((volatile int *)ctx->pinned)[1];
             bl_cur = 0;
@@ -1711,7 +1711,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
                                                                                 xtotal);
       INL_CUDA(cudaGetLastError());
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, f.counts, 48, cudaMemcpyDeviceToHost, st));
-      INL_CUDA(cudaStreamSynchronize(st));
+      ctx_sync(ctx);
       nF = ((volatile int *)ctx->pinned)[0];
       const unsigned long long tot = *(volatile unsigned long long *)((int *)ctx->pinned + 10);
       if (tot == 0) break;
@@ -1722,7 +1722,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, next, n + 1, ncclUint8, ncclMax);
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, next + n, 1, cudaMemcpyDeviceToHost, st));
-      INL_CUDA(cudaStreamSynchronize(st));
+      ctx_sync(ctx);
       if (*(volatile uint8_t *)ctx->pinned == 0) break;
       INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
       k_bfs_apply<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(next, n, level, bm, L, G.row_begin,

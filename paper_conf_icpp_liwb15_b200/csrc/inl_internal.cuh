@@ -253,5 +253,14 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
             inl_stats *stats, bool symmetric);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);
+// Wait for the ctx stream.  NCCL ranks poll instead (ncclCommGetAsyncError): a failed peer or
+// a stuck collective surfaces as INL_ERR_NCCL (communicator aborted) instead of a hang; the
+// limit is INL_NCCL_TIMEOUT_S seconds (default 600).  api.cu.
+void ctx_sync(inl_ctx ctx);
+// NVTX range around a C-ABI call (visible in nsys / ncu timelines; free without a tool)
+struct NvtxRange {
+  explicit NvtxRange(const char *name);
+  ~NvtxRange();
+};
 void sssp_graph_free(void *g);  // frontier.cu
 }  // namespace inl

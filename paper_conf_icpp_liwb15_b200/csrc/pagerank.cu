@@ -191,7 +191,7 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
   std::vector<int32_t> at(gb.size());
   for (size_t i = 0; i < gb.size(); ++i)
     INL_CUDA(cudaMemcpyAsync(&at[i], pos + gb[i], sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-  INL_CUDA(cudaStreamSynchronize(st));
+  ctx_sync(ctx);
   int64_t bck = 1;
   for (size_t i = 0; i < gb.size(); i += 2) bck = std::max<int64_t>(bck, (int64_t)at[i + 1] - at[i]);
   p->pr_bc = bck;
@@ -255,7 +255,7 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
   if (K > 1 && p->n_items > 0) {
     std::vector<WorkItem> h(p->n_items), o;
     INL_CUDA(cudaMemcpyAsync(h.data(), p->items.p, sizeof(WorkItem) * h.size(), cudaMemcpyDeviceToHost, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
     o.reserve(h.size());
     for (int k = 0; k < K; ++k) {
       p->pr_iofs[k] = (int64_t)o.size();
@@ -265,7 +265,7 @@ static void pr_compact(inl_ctx ctx, inl_plan p, const int32_t *od, int64_t B, in
     INL_CHECK(o.size() == h.size(), "pagerank: sub-block item split lost items");
     WorkItem *d = (WorkItem *)p->pr_items.get(sizeof(WorkItem) * o.size());
     INL_CUDA(cudaMemcpyAsync(d, o.data(), sizeof(WorkItem) * o.size(), cudaMemcpyHostToDevice, st));
-    INL_CUDA(cudaStreamSynchronize(st));
+    ctx_sync(ctx);
   }
   p->pr_od = od;
   p->pr_P = P;

@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 out=gpurun_out/bench_all.txt
 : > $out
-run() { echo "== $*" >> $out; timeout 600 python bench.py --no-e2e --no-cpu-baseline "$@" >> $out 2>>gpurun_out/bench_all.err; }
+run() { echo "== $*" >> $out; timeout 600 python bench.py --no-e2e --no-cpu-baseline --no-context "$@" >> $out 2>>gpurun_out/bench_all.err; }
 run --op spmv
 run --op spmv --thread-only
 run --op sssp --steps 9 --warmup 3
@@ -11,6 +11,6 @@ run --op sssp --steps 9 --warmup 3 --thread-only
 run --op bfs --steps 9 --warmup 3
 run --op bfs --steps 9 --warmup 3 --thread-only
 run --op pagerank --steps 3 --warmup 1
-run --op bfs --scale 26 --steps 4 --warmup 1
+run --op bfs --scale 26 --steps 8 --warmup 3
 run --op bc --steps 8 --warmup 3
 run --op bc --scale 22 --steps 4 --warmup 3

@@ -1,5 +1,6 @@
-"""compute-sanitizer (memcheck, racecheck, synccheck) over every kernel of the path on small
-inputs (SURVEY §4.3 tests/sanitize): no out-of-bounds access, no shared-memory race."""
+"""compute-sanitizer (memcheck, racecheck, synccheck, initcheck) over every kernel of the path on
+small inputs (SURVEY §4.3 tests/sanitize): no out-of-bounds access, no shared-memory race, no
+barrier misuse, no read of uninitialised device memory."""
 import os
 import shutil
 import subprocess
@@ -11,7 +12,7 @@ pytestmark = pytest.mark.gpu
 HERE = os.path.dirname(os.path.abspath(__file__))
 
 
-@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck", "initcheck"])
 def test_compute_sanitizer(tool):
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
     cmd = [cs, "--tool", tool, "--error-exitcode", "17", "--print-limit", "20"]
