@@ -238,6 +238,25 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
 inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t n_sources, double *bc,
                   inl_stats *stats, inl_plan plan);
 
+/* Tree descendants / heights (§II.C Fig. 3, §III.C) of the tree
+ * below `root` given as its children CSR T (one GPU, whole CSR; every node reachable from
+ * root at most once):
+ *   desc[v]   = 1 + sum_{c child of v} desc[c]     (inl_tree_descendants)
+ *   height[v] = 1 + max_{c child of v} height[c]    (inl_tree_heights; a leaf has height 1)
+ * out [n_global] int64 (device or host), 0 for nodes not reachable from root.
+ * method INL_TREE_FLAT: the paper's flat template (Fig. 3(c)): one thread per node walks up
+ * parent[] (int32 [n_global], parent[root] = -1; required) with atomicAdd / atomicMax into the
+ * ancestors; stats->edges_relaxed = atomics performed (the sum of node depths for descendants).
+ * method INL_TREE_LEVELS: the B200 form of the hierarchical template (Fig. 3(e)) without
+ * nested launches: nodes grouped by level (top-down BFS + radix sort), one launch per level,
+ * deepest first, 8-lane groups pull their node's children; no atomics; parent may be NULL.
+ * stats->iterations = levels, launches = kernels of the method.  Blocks until done. */
+enum { INL_TREE_FLAT = 0, INL_TREE_LEVELS = 1 };
+inl_status inl_tree_descendants(inl_ctx ctx, const inl_csr *T, const int32_t *parent, int64_t root,
+                                int32_t method, int64_t *desc, inl_stats *stats);
+inl_status inl_tree_heights(inl_ctx ctx, const inl_csr *T, const int32_t *parent, int64_t root,
+                            int32_t method, int64_t *height, inl_stats *stats);
+
 /* Kernel timer (measurement only; off by default).  While enabled, every launch of the
  * path's main kernels ("k_gather", "k_gather_thread_only", "k_expand_flat",
  * "k_expand_grid", "k_bfs_bottom_up") is bracketed by CUDA events recorded on the ctx

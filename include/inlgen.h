@@ -82,6 +82,13 @@ int inlgen_graph_values(inlgen_graph g, float *val); /* -1 if the graph has none
 int inlgen_powerlaw_build(int64_t n, int dmin, int dmax, double mean, uint64_t seed, int flags,
                           inlgen_graph *out);
 
+/* Synthetic tree of PAPER.md §III.C: `depth` levels, every non-leaf node
+ * has `outdegree` children, a node below the last level has children with probability
+ * (1/2)^sparsity (the root always).  Level-order ids (root 0, siblings consecutive); the
+ * children CSR is the graph, parent[] (parent[0] = -1) via inlgen_graph_parent. */
+int inlgen_tree_build(int depth, int outdegree, int sparsity, uint64_t seed, inlgen_graph *out);
+int inlgen_graph_parent(inlgen_graph g, int32_t *parent);
+
 /* Per-entry inputs for a (local) CSR whose row 0 is global row `row_begin`.
  * *_host: host arrays.  *_dev: device arrays, asynchronous on `stream`. */
 int inlgen_weights_host(int64_t n_rows, int64_t row_begin, const int64_t *row_ptr,

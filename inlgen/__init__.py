@@ -52,6 +52,8 @@ def lib() -> C.CDLL:
         L.inlgen_graph_from_csr.argtypes = [i64, i64, i64, vp, vp, vp, vp, C.POINTER(vp)]
         L.inlgen_graph_values.argtypes = [vp, vp]
         L.inlgen_powerlaw_build.argtypes = [i64, i32, i32, C.c_double, u64, i32, C.POINTER(vp)]
+        L.inlgen_tree_build.argtypes = [i32, i32, i32, u64, C.POINTER(vp)]
+        L.inlgen_graph_parent.argtypes = [vp, vp]
         L.inlgen_vector_dev.argtypes = [i64, i64, u64, i32, vp, vp]
         _lib = L
     return _lib
@@ -199,6 +201,22 @@ def powerlaw_build(n: int, dmin: int, dmax: int, mean: float, seed: int = SEED_G
     g = C.c_void_p()
     _check(lib().inlgen_powerlaw_build(n, dmin, dmax, mean, seed, 0, C.byref(g)), "inlgen_powerlaw_build")
     return _host_graph(g, SYMMETRIC)
+
+
+SEED_TREE = 6
+
+
+def tree_build(depth: int, outdegree: int, sparsity: int = 0, seed: int = SEED_TREE) -> HostGraph:
+    """Synthetic tree of PAPER.md §III.C (depth levels, outdegree, sparsity): the children CSR
+    (level-order ids, root 0) with .parent (parent[0] = -1)."""
+    g = C.c_void_p()
+    _check(lib().inlgen_tree_build(depth, outdegree, sparsity, seed, C.byref(g)), "inlgen_tree_build")
+    n_global = _info(g)[0]
+    par = np.empty(max(n_global, 1), dtype=np.int32)
+    _check(lib().inlgen_graph_parent(g, par.ctypes.data), "inlgen_graph_parent")
+    h = _host_graph(g)
+    h.parent = par[:n_global]
+    return h
 
 
 # PAPER.md P5@12491-13052: CiteSeer, 434,102 nodes, "16 million edges", degree 1..1,188, mean 73.9

@@ -217,6 +217,7 @@ extern "C" void inlgen_graph_free(inlgen_graph g) {
     free(g->col_idx);
     free(g->out_degree);
     free(g->val);
+    free(g->parent);
   }
   free(g);
 }

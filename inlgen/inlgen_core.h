@@ -34,7 +34,8 @@ enum {
   IG_STREAM_RELABEL = 5,
   IG_STREAM_SOURCE = 6,
   IG_STREAM_PL_DEGREE = 7,  /* power-law degree sequence (loader.cpp) */
-  IG_STREAM_PL_SHUFFLE = 8  /* its stub shuffle */
+  IG_STREAM_PL_SHUFFLE = 8, /* its stub shuffle */
+  IG_STREAM_TREE = 9        /* synthetic trees: does node v have children */
 };
 
 typedef struct { uint32_t v[4]; } ig_u32x4;

@@ -13,6 +13,7 @@ struct inlgen_graph_s {
   int32_t *col_idx;    /* [nnz] */
   int32_t *out_degree; /* [n_global] or NULL */
   float *val;          /* [nnz] or NULL (loaded matrices with values; host graphs only) */
+  int32_t *parent;     /* [n_global] or NULL (trees from inlgen_tree_build) */
 };
 
 #ifdef __cplusplus

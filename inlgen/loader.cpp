@@ -370,3 +370,68 @@ static int powerlaw_once(int64_t n, int dmin, int dmax, double mean, uint64_t se
   orient(e, INLGEN_SYMMETRIC);
   return build_csr(e, n, n, false, false, out);
 }
+
+// ---- synthetic trees (§III.C P11@8056: "three parameters: tree
+// depth, node outdegree and sparsity ... All non-leaf nodes have the same number of children,
+// which is given by the node outdegree parameter.  The probability rho of the non-leaf nodes
+// having children is defined as rho = (1/2)^sparsity" — reading R14: the garbled formula is
+// (1/2)^sparsity; the root always has children; `depth` counts levels, so the leaves of a
+// regular tree are at level depth-1 and the flat kernel's atomics are d + 2d^2 + 3d^3 at
+// depth 4, Fig. 7(c)).  Node ids are level order (BFS numbering): the root is 0 and a node's
+// children are consecutive.  Children CSR in row_ptr / col_idx; parent[] via inlgen_graph_parent
+// (parent[0] = -1).  Node v (below the last level) has children iff a Philox draw keyed by
+// (seed, v) is below rho * 2^32.
+extern "C" int inlgen_tree_build(int depth, int outdegree, int sparsity, uint64_t seed, inlgen_graph *out) {
+  if (!out || depth < 1 || outdegree < 1 || sparsity < 0 || sparsity > 31) {
+    inlgen_set_error("inlgen_tree_build: bad argument (depth >= 1, outdegree >= 1, sparsity in [0, 31])");
+    return -1;
+  }
+  const uint64_t thr = sparsity == 0 ? 0x100000000ull : (0x100000000ull >> sparsity);  // rho * 2^32
+  std::vector<int64_t> rp(1, 0);
+  std::vector<int32_t> col, par(1, -1);
+  int64_t lo = 0, hi = 1;  // the current level's nodes
+  for (int lev = 0; lev < depth; ++lev) {
+    for (int64_t v = lo; v < hi; ++v) {
+      const bool kids = lev + 1 < depth && (v == 0 || (uint64_t)ig_draw(seed, IG_STREAM_TREE, (uint64_t)v, 0, 0) < thr);
+      if (kids) {
+        if ((int64_t)par.size() + outdegree >= INT32_MAX) {
+          inlgen_set_error("inlgen_tree_build: more than 2^31 nodes");
+          return -1;
+        }
+        for (int c = 0; c < outdegree; ++c) {
+          col.push_back((int32_t)par.size());
+          par.push_back((int32_t)v);
+        }
+      }
+      rp.push_back((int64_t)col.size());
+    }
+    lo = hi;
+    hi = (int64_t)par.size();
+  }
+  const int64_t n = (int64_t)par.size();
+  inlgen_graph g = (inlgen_graph)calloc(1, sizeof(*g));
+  if (!g) return -2;
+  g->n_global = g->n_rows = n;
+  g->nnz = (int64_t)col.size();
+  g->row_ptr = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n + 1));
+  g->col_idx = (int32_t *)malloc(sizeof(int32_t) * (col.empty() ? 1 : col.size()));
+  g->parent = (int32_t *)malloc(sizeof(int32_t) * (size_t)n);
+  if (!g->row_ptr || !g->col_idx || !g->parent) {
+    inlgen_graph_free(g);
+    return -2;
+  }
+  memcpy(g->row_ptr, rp.data(), sizeof(int64_t) * (size_t)(n + 1));
+  if (!col.empty()) memcpy(g->col_idx, col.data(), sizeof(int32_t) * col.size());
+  memcpy(g->parent, par.data(), sizeof(int32_t) * (size_t)n);
+  *out = g;
+  return 0;
+}
+
+extern "C" int inlgen_graph_parent(inlgen_graph g, int32_t *parent) {
+  if (!g || !parent || !g->parent || g->on_device) {
+    inlgen_set_error("inlgen_graph_parent: not a tree from inlgen_tree_build");
+    return -1;
+  }
+  memcpy(parent, g->parent, sizeof(int32_t) * (size_t)g->n_global);
+  return 0;
+}

@@ -30,6 +30,8 @@ def lib() -> C.CDLL:
         L.orc_sssp_dijkstra.argtypes = [i64, vp, vp, vp, i64, vp]
         L.orc_bfs.argtypes = [i64, vp, vp, i64, vp]
         L.orc_bc.argtypes = [i64, vp, vp, vp, i64, vp]
+        L.orc_tree_descendants.argtypes = [i64, vp, vp, i64, vp]
+        L.orc_tree_heights.argtypes = [i64, vp, vp, i64, vp]
         _lib = L
     return _lib
 
@@ -136,4 +138,24 @@ def bc(row_ptr, col_idx, sources=None) -> np.ndarray:
     out = np.empty(n, dtype=np.float64)
     _rc(lib().orc_bc(n, prp, pci, src.ctypes.data if src.size else 0, len(src), out.ctypes.data if n else 0),
         "orc_bc")
+    return out
+
+
+def tree_descendants(row_ptr, col_idx, root=0) -> np.ndarray:
+    """desc[v] = 1 + sum of desc over v's children (children CSR), int64."""
+    rp, prp = _a(row_ptr, np.int64)
+    ci, pci = _a(col_idx, np.int32)
+    n = len(rp) - 1
+    out = np.empty(n, dtype=np.int64)
+    _rc(lib().orc_tree_descendants(n, prp, pci, root, out.ctypes.data if n else 0), "orc_tree_descendants")
+    return out
+
+
+def tree_heights(row_ptr, col_idx, root=0) -> np.ndarray:
+    """height[v] = 1 + max height over v's children (a leaf: 1), int64."""
+    rp, prp = _a(row_ptr, np.int64)
+    ci, pci = _a(col_idx, np.int32)
+    n = len(rp) - 1
+    out = np.empty(n, dtype=np.int64)
+    _rc(lib().orc_tree_heights(n, prp, pci, root, out.ctypes.data if n else 0), "orc_tree_heights")
     return out

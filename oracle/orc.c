@@ -233,3 +233,73 @@ int orc_bc(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int6
   free(delta);
   return 0;
 }
+
+/* Tree descendants and heights — PAPER.md §II.C (P5@5170-7323, Fig. 3(a)): "the recursive
+ * computation of the number of descendants in a tree ... the descendants array, which stores
+ * the number of descendants of all nodes, is initialized to all 1s (that is, every node is a
+ * descendant of itself)"; Tree Heights is "similar code" (P5@11250).  Fig. 3(a)'s recursion
+ *   descendants(v) = 1 + sum_{c child of v} descendants(c)
+ *   height(v)      = 1 + max_{c child of v} height(c)   (a leaf: 1; reading R14)
+ * evaluated without recursion: nodes in BFS order from the root, then in reverse, so every
+ * child is finished before its parent.  Input: the children CSR; nodes not reachable from
+ * `root` get 0. */
+static int orc_tree_order(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t root,
+                          int64_t *order, int64_t *count) {
+  if (n <= 0 || root < 0 || root >= n) return -1;
+  char *seen = (char *)calloc((size_t)n, 1);
+  if (!seen) return -2;
+  int64_t head = 0, tail = 0;
+  order[tail++] = root;
+  seen[root] = 1;
+  while (head < tail) {
+    const int64_t v = order[head++];
+    for (int64_t k = row_ptr[v]; k < row_ptr[v + 1]; ++k) {
+      const int64_t c = col_idx[k];
+      if (c < 0 || c >= n || seen[c]) { free(seen); return -1; } /* not a tree */
+      seen[c] = 1;
+      order[tail++] = c;
+    }
+  }
+  free(seen);
+  *count = tail;
+  return 0;
+}
+
+int orc_tree_descendants(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t root,
+                         int64_t *desc) {
+  if (n < 0 || (n > 0 && (!row_ptr || !desc))) return -1;
+  if (n == 0) return 0;
+  int64_t *order = (int64_t *)malloc(sizeof(int64_t) * (size_t)n), cnt = 0;
+  if (!order) return -2;
+  const int rc = orc_tree_order(n, row_ptr, col_idx, root, order, &cnt);
+  if (rc) { free(order); return rc; }
+  for (int64_t v = 0; v < n; ++v) desc[v] = 0;
+  for (int64_t j = cnt - 1; j >= 0; --j) {
+    const int64_t v = order[j];
+    int64_t s = 1;
+    for (int64_t k = row_ptr[v]; k < row_ptr[v + 1]; ++k) s += desc[col_idx[k]];
+    desc[v] = s;
+  }
+  free(order);
+  return 0;
+}
+
+int orc_tree_heights(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t root,
+                     int64_t *height) {
+  if (n < 0 || (n > 0 && (!row_ptr || !height))) return -1;
+  if (n == 0) return 0;
+  int64_t *order = (int64_t *)malloc(sizeof(int64_t) * (size_t)n), cnt = 0;
+  if (!order) return -2;
+  const int rc = orc_tree_order(n, row_ptr, col_idx, root, order, &cnt);
+  if (rc) { free(order); return rc; }
+  for (int64_t v = 0; v < n; ++v) height[v] = 0;
+  for (int64_t j = cnt - 1; j >= 0; --j) {
+    const int64_t v = order[j];
+    int64_t h = 0;
+    for (int64_t k = row_ptr[v]; k < row_ptr[v + 1]; ++k)
+      if (height[col_idx[k]] > h) h = height[col_idx[k]];
+    height[v] = 1 + h;
+  }
+  free(order);
+  return 0;
+}

@@ -52,6 +52,16 @@ int orc_bfs(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t s
 int orc_bc(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, const int64_t *sources,
            int64_t n_sources, double *bc);
 
+/* Tree descendants / heights (§II.C Fig. 3(a), §III.C) over the
+ * children CSR of a tree rooted at `root`:
+ *   desc[v]   = 1 + sum_{c child of v} desc[c]          (every node descends from itself)
+ *   height[v] = 1 + max_{c child of v} height[c]         (a leaf has height 1; reading R14)
+ * int64; nodes not reachable from root get 0.  -1 if the CSR is not a tree below root. */
+int orc_tree_descendants(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t root,
+                         int64_t *desc);
+int orc_tree_heights(int64_t n, const int64_t *row_ptr, const int32_t *col_idx, int64_t root,
+                     int64_t *height);
+
 #ifdef __cplusplus
 }
 #endif

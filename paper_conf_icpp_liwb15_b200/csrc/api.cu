@@ -775,4 +775,36 @@ inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t
   });
 }
 
+static inl_status tree_entry(inl_ctx ctx, const inl_csr *T, const int32_t *parent, int64_t root, int32_t method,
+                             int64_t *out, inl_stats *stats, bool heights) {
+  if (!ctx) return fail(nullptr, INL_ERR_INVALID_ARGUMENT, "ctx is NULL");
+  return guarded(ctx, [&] {
+    check_csr(T);
+    INL_CHECK(T->row_begin == 0 && T->n_rows == T->n_global, "tree: one GPU, the whole children CSR");
+    INL_CHECK(T->n_global == 0 || (root >= 0 && root < T->n_global), "tree: root out of range");
+    INL_CHECK(T->n_global == 0 || out != nullptr, "tree: output is NULL");
+    INL_CHECK(method == INL_TREE_FLAT || method == INL_TREE_LEVELS, "tree: unknown method");
+    INL_CHECK(method != INL_TREE_FLAT || T->n_global == 0 || parent != nullptr, "tree: INL_TREE_FLAT needs parent[]");
+    DeviceGuard g(ctx->device);
+    inl_csr d = device_csr(ctx, T);
+    const int32_t *dpar = stage_in(ctx, ctx->h_od, parent, T->n_global);
+    StagedOut<int64_t> o = stage_out(ctx->h_y, out, T->n_global);
+    tree_run(ctx, d, dpar, root, method, heights, o.dev, stats);
+    finish_out(ctx, o);
+    ctx_sync(ctx);
+  });
+}
+
+inl_status inl_tree_descendants(inl_ctx ctx, const inl_csr *T, const int32_t *parent, int64_t root, int32_t method,
+                                int64_t *desc, inl_stats *stats) {
+  NvtxRange nvtx_("inl_tree_descendants");
+  return tree_entry(ctx, T, parent, root, method, desc, stats, false);
+}
+
+inl_status inl_tree_heights(inl_ctx ctx, const inl_csr *T, const int32_t *parent, int64_t root, int32_t method,
+                            int64_t *height, inl_stats *stats) {
+  NvtxRange nvtx_("inl_tree_heights");
+  return tree_entry(ctx, T, parent, root, method, height, stats, true);
+}
+
 }  // extern "C"

@@ -153,6 +153,7 @@ struct inl_ctx_s {
   inl::DevBuf s_loop;                                  // loopback allreduce scratch
   inl::DevBuf s_pad;                                   // padded replicated vectors (P > 1)
   inl::DevBuf s_bu;                                    // BFS bottom-up worklists
+  inl::DevBuf s_h;                                     // tree levels (tree.cu)
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
@@ -248,6 +249,9 @@ constexpr int kTemplateFlags = INL_BINS_TPL_DUAL_QUEUE | INL_BINS_TPL_DBUF_GLOBA
 bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *val, const float *x, float *y);
 // colblock.cu: builds `cb` for the column space `cols` (raw ids in [0, ncols), CSR order)
 void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool sort_rows = false);
+// tree.cu: descendants (heights = false) or heights of the tree below `root`
+void tree_run(inl_ctx ctx, const inl_csr &T, const int32_t *parent, int64_t root, int method, bool heights,
+              int64_t *out, inl_stats *stats);
 // bc.cu
 void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
             inl_stats *stats, bool symmetric);

@@ -29,6 +29,8 @@ BINS_SSSP_DEVLOOP = 4
 BINS_TPL_DUAL_QUEUE = 8
 BINS_TPL_DBUF_GLOBAL = 16
 BINS_TPL_DBUF_SHARED = 32
+TREE_FLAT = 0    # the paper's flat template: thread per node, atomics up the parent chain
+TREE_LEVELS = 1  # level-synchronous pull (B200 form of the hierarchical template)
 
 
 class InlError(RuntimeError):
@@ -97,11 +99,14 @@ def lib() -> C.CDLL:
         L.inl_sssp.argtypes = [vp, C.POINTER(CsrT), vp, i64, vp, C.POINTER(StatsT), vp]
         L.inl_bfs.argtypes = [vp, C.POINTER(CsrT), i64, vp, C.POINTER(StatsT), vp]
         L.inl_bc.argtypes = [vp, C.POINTER(CsrT), vp, i64, vp, C.POINTER(StatsT), vp]
+        L.inl_tree_descendants.argtypes = [vp, C.POINTER(CsrT), vp, i64, i32, vp, C.POINTER(StatsT)]
+        L.inl_tree_heights.argtypes = [vp, C.POINTER(CsrT), vp, i64, i32, vp, C.POINTER(StatsT)]
         L.inl_ktimer_enable.argtypes = [vp, i32]
         L.inl_ktimer_read.argtypes = [vp, C.c_char_p, C.POINTER(i64), C.POINTER(C.c_double)]
         for f in ("inl_ctx_create", "inl_ctx_set_stream", "inl_ctx_destroy", "inl_partition_rows",
                   "inl_nccl_unique_id", "inl_comm_init", "inl_loop_create", "inl_loop_destroy",
-                  "inl_comm_init_loopback", "inl_spmv_allgather", "inl_plan_create", "inl_plan_get_info",
+                  "inl_comm_init_loopback", "inl_spmv_allgather", "inl_tree_descendants", "inl_tree_heights",
+                  "inl_plan_create", "inl_plan_get_info",
                   "inl_plan_destroy", "inl_csr_validate", "inl_spmv", "inl_pagerank", "inl_sssp", "inl_bfs",
                   "inl_ktimer_enable", "inl_ktimer_read"):
             getattr(L, f).restype = C.c_int
@@ -362,3 +367,22 @@ def bc(ctx: Ctx, G: Csr, sources, out, plan: Plan | None = None) -> dict:
                         C.byref(st), _plan_handle(plan)), ctx)
     return {"iterations": st.iterations, "frontier_total": st.frontier_total, "launches": st.launches,
             "host_syncs": st.host_syncs}
+
+
+def _tree(fn, ctx, T, parent, root, out, method):
+    ctx.sync_stream()
+    s = T.struct()
+    st = StatsT()
+    _check(fn(ctx.handle, C.byref(s), _ptr(parent), int(root), int(method), _ptr(out), C.byref(st)), ctx)
+    return {"levels": st.iterations, "atomics": st.edges_relaxed, "launches": st.launches,
+            "host_syncs": st.host_syncs}
+
+
+def tree_descendants(ctx: Ctx, T: Csr, parent, out, root: int = 0, method: int = TREE_LEVELS) -> dict:
+    """desc[v] = 1 + sum of desc over v's children (§II.C Fig. 3); out int64 [n]."""
+    return _tree(lib().inl_tree_descendants, ctx, T, parent, root, out, method)
+
+
+def tree_heights(ctx: Ctx, T: Csr, parent, out, root: int = 0, method: int = TREE_LEVELS) -> dict:
+    """height[v] = 1 + max height over v's children, a leaf 1 (reading R14); out int64 [n]."""
+    return _tree(lib().inl_tree_heights, ctx, T, parent, root, out, method)

@@ -1,0 +1,124 @@
+"""CPU pins of the tree oracle (§II.C Fig. 3, §III.C) and of the
+tree generator's reading of the garbled sparsity formula (R14).
+
+* Closed forms on regular trees: a node at level k of a depth-D tree with outdegree d has
+  (d^(D-k) - 1) / (d - 1) descendants (itself included) and height D - k (a leaf: 1).
+* Brute force on random trees (random parents, not level-ordered): descendants by walking every
+  node's ancestor chain, heights by the longest ancestor chain above each leaf.
+* The paper's Fig. 7(c) "Atomic" column for the flat kernel = the sum of node depths
+  = sum(desc) - n: d + 2d^2 + 3d^3 on a regular depth-4 tree (0.10 m at d = 32, 0.79 m at 64,
+  6.32 m at 128, 50.4 m at 256, 403 m at 512), and the sparsity rows at d = 512 (26.0 m,
+  6.70 m, 1.68 m for sparsity 2, 3, 4) within the spread of one random tree, which pins
+  rho = (1/2)^sparsity with the root always expanded.
+"""
+import numpy as np
+import pytest
+
+import inlgen
+import oracle
+
+
+def children_csr(parent):
+    n = len(parent)
+    kids = [[] for _ in range(n)]
+    for v, p in enumerate(parent):
+        if p >= 0:
+            kids[p].append(v)
+    rp = np.zeros(n + 1, np.int64)
+    for v in range(n):
+        rp[v + 1] = rp[v] + len(kids[v])
+    ci = np.array([c for k in kids for c in k], dtype=np.int32)
+    return rp, ci
+
+
+def brute(parent):
+    n = len(parent)
+    desc = np.zeros(n, np.int64)
+    depth = np.zeros(n, np.int64)
+    for v in range(n):
+        u, d = v, 0
+        while u >= 0:
+            desc[u] += 1
+            u = parent[u]
+            d += 1
+        depth[v] = d - 1
+    has_kid = np.zeros(n, bool)
+    for v in range(n):
+        if parent[v] >= 0:
+            has_kid[parent[v]] = True
+    height = np.zeros(n, np.int64)
+    for v in range(n):
+        if has_kid[v]:
+            continue
+        u, h = v, 1
+        while u >= 0:
+            height[u] = max(height[u], h)
+            u = parent[u]
+            h += 1
+    return desc, height, depth
+
+
+@pytest.mark.parametrize("D,d", [(1, 5), (2, 1), (3, 2), (4, 3), (5, 4), (4, 32)])
+def test_regular_tree_closed_forms(D, d):
+    t = inlgen.tree_build(D, d, 0)
+    desc = oracle.tree_descendants(t.row_ptr, t.col_idx, 0)
+    height = oracle.tree_heights(t.row_ptr, t.col_idx, 0)
+    lvl_start = 0
+    for k in range(D):
+        cnt = d ** k
+        want_desc = (d ** (D - k) - 1) // (d - 1) if d > 1 else D - k
+        assert np.all(desc[lvl_start:lvl_start + cnt] == want_desc), k
+        assert np.all(height[lvl_start:lvl_start + cnt] == D - k), k
+        lvl_start += cnt
+    assert lvl_start == t.n_global
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_trees_brute_force(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 400))
+    perm = rng.permutation(n)  # node ids not in level order; root = perm[0]
+    parent = np.full(n, -1, np.int64)
+    for i in range(1, n):
+        parent[perm[i]] = perm[int(rng.integers(0, i))]
+    rp, ci = children_csr(parent)
+    root = int(perm[0])
+    desc, height, _ = brute(parent)
+    assert np.array_equal(oracle.tree_descendants(rp, ci, root), desc)
+    assert np.array_equal(oracle.tree_heights(rp, ci, root), height)
+
+
+def test_unreachable_nodes_and_not_a_tree():
+    rp, ci = children_csr(np.array([-1, 0, 0, -1, 3]))  # 3..4: another tree
+    assert oracle.tree_descendants(rp, ci, 0).tolist() == [3, 1, 1, 0, 0]
+    assert oracle.tree_heights(rp, ci, 3).tolist() == [0, 0, 0, 2, 1]
+    # node 2 reachable twice: not a tree
+    rp = np.array([0, 2, 3, 3], np.int64)
+    ci = np.array([1, 2, 2], np.int32)
+    with pytest.raises(RuntimeError):
+        oracle.tree_descendants(rp, ci, 0)
+
+
+@pytest.mark.parametrize("d,paper", [(32, 0.10e6), (64, 0.79e6)])
+def test_fig7c_flat_atomics_regular(d, paper):
+    t = inlgen.tree_build(4, d, 0)
+    desc = oracle.tree_descendants(t.row_ptr, t.col_idx, 0)
+    atomics = int(desc.sum()) - t.n_global  # = sum of depths
+    assert atomics == d + 2 * d * d + 3 * d ** 3
+    assert abs(atomics - paper) / paper < 0.01
+    for dd, p in ((128, 6.32e6), (256, 50.4e6), (512, 403e6)):  # the formula at the larger sizes
+        assert abs(dd + 2 * dd * dd + 3 * dd ** 3 - p) / p < 0.005
+
+
+@pytest.mark.parametrize("sparsity,paper", [(2, 26.0e6), (3, 6.70e6), (4, 1.68e6)])
+def test_fig7c_sparsity_rows(sparsity, paper):
+    t = inlgen.tree_build(4, 512, sparsity)
+    rp, ci = t.row_ptr, t.col_idx
+    desc = oracle.tree_descendants(rp, ci, 0)
+    atomics = int(desc.sum()) - t.n_global
+    rho = 0.5 ** sparsity
+    expect = 512 + 2 * rho * 512 ** 2 + 3 * rho ** 2 * 512 ** 3
+    assert abs(atomics - expect) / expect < 0.08      # one random tree around its mean (512 coin flips at level 1)
+    assert abs(atomics - paper) / paper < 0.08        # and near the paper's printed value
+    deg = np.diff(rp)
+    assert set(np.unique(deg).tolist()) <= {0, 512}   # every non-leaf has outdegree children
