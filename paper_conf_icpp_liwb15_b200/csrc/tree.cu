@@ -164,8 +164,8 @@ void tree_run(inl_ctx ctx, const inl_csr &T, const int32_t *parent, int64_t root
     size_t need = 0;
     INL_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, need, kb, vb, (int)n, 0, 32, st));
     INL_CUDA(cub::DeviceRadixSort::SortPairs(ctx->s_tmp.get(need), need, kb, vb, (int)n, 0, 32, st));
-    // level sizes (a histogram; depth = bst.iterations + 1 levels) -> boundaries on the host
-    const int depth = bst.iterations + 1;
+    // level sizes (a histogram over the BFS's levels 0 .. iterations-1) -> boundaries on the host
+    const int depth = bst.iterations > 0 ? bst.iterations : 1;
     unsigned long long *hist = (unsigned long long *)ctx->s_g.get(sizeof(unsigned long long) * (size_t)(depth + 1));
     INL_CUDA(cudaMemsetAsync(hist, 0, sizeof(unsigned long long) * (size_t)(depth + 1), st));
     k_level_hist<<<tgrid(n, ctx->num_sms), 256, depth <= kHistSmem ? sizeof(unsigned int) * depth : 0, st>>>(
@@ -195,7 +195,7 @@ void tree_run(inl_ctx ctx, const inl_csr &T, const int32_t *parent, int64_t root
     unsigned long long a = 0;
     INL_CUDA(cudaMemcpyAsync(&a, atomics, sizeof a, cudaMemcpyDeviceToHost, st));
     ctx_sync(ctx);
-    stats->iterations = bst.iterations + 1;  // levels
+    stats->iterations = bst.iterations;      // levels
     stats->edges_relaxed = (int64_t)a;       // atomics (INL_TREE_FLAT), 0 for INL_TREE_LEVELS
     stats->frontier_total = bst.frontier_total;
     stats->launches = launches;
