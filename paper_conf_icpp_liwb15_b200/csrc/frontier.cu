@@ -42,6 +42,10 @@ namespace {
 
 constexpr int NT = 256;
 constexpr int NW = NT / 32;
+// resident CTAs per SM the expansion kernels are compiled for (register cap 65536 / (NT * it))
+#ifndef INL_EXPAND_MINB
+#define INL_EXPAND_MINB 1
+#endif
 
 __device__ __forceinline__ void push(int32_t *q, int *cnt, int32_t v) {
   cg::coalesced_group g = cg::coalesced_threads();
@@ -424,7 +428,7 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
 constexpr int kEdgesPerThread = 8;
 
 template <class Op>
-__global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
+__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
@@ -534,7 +538,7 @@ __global__ void __launch_bounds__(NT) k_expand_flat(ExpandArgs a, Op op) {
 // Grid bin (dbuf-global, P5@2721): pieces of grid_chunk edges of the large-degree
 // frontier vertices, one CTA per piece (grid-stride); each thread keeps 8 edges in flight.
 template <class Op>
-__global__ void __launch_bounds__(NT) k_expand_grid(ExpandArgs a, Op op) {
+__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_grid(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
