@@ -1,7 +1,8 @@
 """world_size-2 CPU tests (gloo) of the multi-GPU row-block path.
 
-The product's N > 1 path is CUDA + NCCL (frontier.cu / pagerank.cu DIST mode); what
-can run here is its host side — the NCCL unique-id bootstrap through libinl and
+The product's N > 1 path itself (libinl's row-block kernels and its exchange, NCCL or the
+one-device loopback communicator) runs under oracle parity in tests/test_gpu_loopback.py
+(P = 2, 3, 8 on one B200).  What can run here, without a GPU, is its host side — the NCCL unique-id bootstrap through libinl and
 torch.distributed, the row-block partition (inl_partition_rows) and per-rank CSR
 slices (inlgen row ranges) — and step-by-step models of the three exchange
 protocols, with gloo standing in for NCCL, checked against the single-process
