@@ -123,6 +123,10 @@ typedef struct {
   int64_t frontier_total; /* sum of frontier sizes over the iterations */
   int64_t launches;       /* kernels the call launched (memsets and copies excluded) */
   int64_t host_syncs;     /* host <-> device round trips of the iteration loop */
+  int64_t exchange_bytes; /* P > 1: bytes this rank moved through the exchange:
+                             collectives by the ring model (allreduce 2(P-1)/P * size, allgather
+                             (P-1)/P * size); NEXT-1 peer-memory exchange: 4 B per remote atomic
+                             (counted on the device) + the peers' bitmap words read */
 } inl_stats;
 
 /* Plan summary (for tests and the bench; counts per bin). */

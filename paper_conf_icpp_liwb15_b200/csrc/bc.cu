@@ -359,6 +359,7 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
     stats->frontier_total = ftotal;
     stats->launches = launches;
     stats->host_syncs = syncs;
+    stats->exchange_bytes = 0;
   }
 }
 

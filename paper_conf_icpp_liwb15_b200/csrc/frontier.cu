@@ -98,6 +98,7 @@ struct SsspOp {
   uint32_t *const *xc = nullptr;   // [P] owners' changed bitmaps of this round
   int64_t B = 0;
   unsigned int *nimp = nullptr;
+  unsigned long long *xops = nullptr;  // remote atomics issued (the exchange volume)
   __device__ __forceinline__ bool xrelax(int32_t v, uint32_t nd) const {
     uint32_t *o = xd[v / B];
     if (o != dist) atomicMin(dist + v, nd);  // keep the local filter tight
@@ -113,7 +114,10 @@ struct SsspOp {
   }
   __device__ __forceinline__ void improve(int32_t v, uint32_t nd, int32_t *q, int *cnt) const {
     if (xd) {
-      if (xrelax(v, nd)) atomicAdd(nimp, 1u);
+      const bool r = xd[v / B] != dist;
+      const bool imp = xrelax(v, nd);
+      if (imp) atomicAdd(nimp, 1u);
+      if (r) atomicAdd(xops, imp ? 2ull : 1ull);
       return;
     }
     const uint32_t old = atomicMin(dist + v, nd);
@@ -147,12 +151,23 @@ struct SsspOp {
 #pragma unroll
     for (int j = 0; j < K; ++j) dv[j] = in[j] ? dist[vv[j]] : 0u;
     if (xd) {  // NEXT-1: improvements go to the owners
-      unsigned c = 0;
+      unsigned c = 0, rem = 0;
 #pragma unroll
       for (int j = 0; j < K; ++j)
-        if (nd[j] < dv[j] && xrelax(vv[j], nd[j])) ++c;
-      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-      if ((threadIdx.x & 31) == 0 && c) atomicAdd(nimp, c);
+        if (nd[j] < dv[j]) {
+          const bool r = xd[vv[j] / B] != dist;
+          const bool imp = xrelax(vv[j], nd[j]);
+          c += imp;
+          rem += r ? 1u + (imp ? 1u : 0u) : 0u;  // the remote atomicMin (+ the changed bit)
+        }
+      for (int o = 16; o > 0; o >>= 1) {
+        c += __shfl_xor_sync(0xffffffffu, c, o);
+        rem += __shfl_xor_sync(0xffffffffu, rem, o);
+      }
+      if ((threadIdx.x & 31) == 0) {
+        if (c) atomicAdd(nimp, c);
+        if (rem) atomicAdd(xops, (unsigned long long)rem);
+      }
       return;
     }
 #pragma unroll
@@ -196,6 +211,8 @@ struct BfsOp {
   // loopback), during the expansion itself — no byte map, no allreduce
   uint32_t *const *xtab = nullptr;   // [P] owners' bitmaps of this level
   int64_t B = 0;                     // row block
+  const uint32_t *xself = nullptr;   // this rank's own bitmap (local sets are not exchange)
+  unsigned long long *xops = nullptr;  // remote atomics issued
   __device__ __forceinline__ void xset(int32_t v) const {
     atomicOr(xtab[v / B] + (v >> 5), 1u << (v & 31));
   }
@@ -206,6 +223,7 @@ struct BfsOp {
   __device__ __forceinline__ void visit(int32_t v, int32_t *q, int *cnt) const {
     if (!enqueue && xtab) {
       xset(v);
+      if (xtab[v / B] != xself) atomicAdd(xops, 1ull);
     } else if (enqueue) {
       const uint32_t bit = 1u << (v & 31);
       const uint32_t old = atomicOr(bitmap + (v >> 5), bit);
@@ -236,9 +254,15 @@ struct BfsOp {
       if (!((bw[j] >> (vv[j] & 31)) & 1u)) cand |= 1u << j;
     if (!enqueue) {
       if (xtab) {
+        unsigned rem = 0;
 #pragma unroll
         for (int j = 0; j < K; ++j)
-          if ((cand >> j) & 1u) xset(vv[j]);
+          if ((cand >> j) & 1u) {
+            xset(vv[j]);
+            rem += xtab[vv[j] / B] != xself;
+          }
+        for (int o = 16; o > 0; o >>= 1) rem += __shfl_xor_sync(0xffffffffu, rem, o);
+        if ((threadIdx.x & 31) == 0 && rem) atomicAdd(xops, (unsigned long long)rem);
         return;
       }
 #pragma unroll
@@ -1119,17 +1143,19 @@ int read_count(inl_ctx ctx, const int *d) {
   return *(volatile int *)ctx->pinned;
 }
 
-void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_t ftotal) {
+// xbytes: exchange bytes counted on the host; the device adds 4 B per remote atomic (counts[12])
+void finish_stats(inl_ctx ctx, FrontierBufs &f, inl_stats *st, int iters, int64_t ftotal, int64_t xbytes = 0) {
   check_overflow(ctx, f);
   if (!st) return;
-  unsigned long long r = 0;
-  INL_CUDA(cudaMemcpyAsync(&r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, ctx->stream));
+  unsigned long long r[3] = {0, 0, 0};  // relaxed (counts[8]), m_f / total (counts[10]), remote atomics (counts[12])
+  INL_CUDA(cudaMemcpyAsync(r, f.relaxed, sizeof r, cudaMemcpyDeviceToHost, ctx->stream));
   ctx_sync(ctx);
   st->iterations = iters;
-  st->edges_relaxed = (int64_t)r;
+  st->edges_relaxed = (int64_t)r[0];
   st->frontier_total = ftotal;
   st->launches = 0;  // host-driven loops: not counted
   st->host_syncs = iters;
+  st->exchange_bytes = xbytes + 4 * (int64_t)r[2];
 }
 
 }  // namespace
@@ -1214,6 +1240,7 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
     stats->frontier_total = (int64_t)hs->ftotal;
     stats->launches = launches;
     stats->host_syncs = syncs;
+    stats->exchange_bytes = 0;
   }
 }
 
@@ -1357,6 +1384,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     stats->frontier_total = (int64_t)hs->ftotal;
     stats->launches = 1 + 4LL * hs->pad;  // init + 4 kernels per step (one graph launch)
     stats->host_syncs = 1;
+    stats->exchange_bytes = 0;
   }
 }
 
@@ -1399,6 +1427,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   const int64_t dlen = (Bk * P + 31) / 32 * 32;      // padded replicated distance vector
   uint32_t *xchg = nullptr, **xtab = nullptr;
   unsigned int *nimp = (unsigned int *)(f.counts + 3);
+  unsigned long long *xops = (unsigned long long *)(f.counts + 12);  // remote atomics (exchange volume)
+  int64_t xbytes = 0;  // exchange bytes of the collectives (ring model)
   if (xsparse) {
     // one exchange buffer: [distances (dlen)] [3 changed-bitmaps (xw each), round r uses r % 3]
     const size_t bytes = sizeof(uint32_t) * ((size_t)dlen + 3 * (size_t)xw);
@@ -1485,8 +1515,10 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       op.xc = xtab + (size_t)(1 + r) * P;
       op.B = Bk;
       op.nimp = nimp;
+      op.xops = xops;
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, nimp, 1, ncclUint32, ncclSum);  // the round's barrier + termination test
+      xbytes += 2 * (int64_t)(P - 1) * 4 / P;
       ++iters;
       INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
       k_sssp_collect_xbits<<<grid_for((G.n_rows + 31) / 32 + 1, ctx->num_sms), 256, 0, st>>>(
@@ -1503,6 +1535,7 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       SsspOp op{D, w, nullptr, D + n, iters, G.row_begin, false, 0, 0xFFFFFFFFu, nullptr, nullptr, nullptr};
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, D, n + 1, ncclUint32, ncclMin);
+      xbytes += 2 * (int64_t)(P - 1) * 4 * (n + 1) / P;
       ++iters;
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, D + n, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
       ctx_sync(ctx);
@@ -1514,11 +1547,13 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
       nF = read_count(ctx, f.counts);
     }
   }
-  if (xsparse)  // replicate: the owners' slices (in place, padded to P equal blocks)
+  if (xsparse) {  // replicate: the owners' slices (in place, padded to P equal blocks)
     comm_allgather(ctx, D + (size_t)ctx->rank * Bk, D, Bk, ncclUint32, nullptr, nullptr);
+    xbytes += 4 * Bk * (int64_t)(P - 1);
+  }
   if (DIST)
     INL_CUDA(cudaMemcpyAsync(dist, D, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, st));
-  finish_stats(ctx, f, stats, iters, ftotal);
+  finish_stats(ctx, f, stats, iters, ftotal, xbytes);
 }
 
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
@@ -1542,6 +1577,8 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   uint32_t *xb = nullptr;
   uint32_t **xtab = nullptr;
   unsigned long long *xtotal = (unsigned long long *)(f.counts + 10);
+  unsigned long long *xops = (unsigned long long *)(f.counts + 12);  // remote atomics (exchange volume)
+  int64_t xbytes = 0;  // exchange bytes counted on the host (collectives, bitmap reads)
   if (xbits && n > 0) {
     // three level buffers (level L writes buffer L % 3; a rank clears buffer (L+1) % 3 before
     // its level-L expansion: every rank read it at level L-2, before the level L-1 barrier, and
@@ -1706,7 +1743,11 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       BfsOp op{bm, level, nullptr, n, L, false, 0};
       op.xtab = xtab + (size_t)buf * P;
       op.B = B;
+      op.xself = xb + (size_t)buf * xw;
+      op.xops = xops;
       expand(ctx, G, b, f, nF, op);
+      // the apply reads every word of the level bitmap outside this rank's block from its owner
+      xbytes += 4 * ((n + 31) / 32 - ((G.row_begin + G.n_rows + 31) / 32 - G.row_begin / 32));
       comm_barrier(ctx);
       INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
       INL_CUDA(cudaMemsetAsync(xtotal, 0, sizeof(unsigned long long), st));
@@ -1725,6 +1766,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       BfsOp op{bm, level, next, n, L, false, 0};
       expand(ctx, G, b, f, nF, op);
       comm_allreduce(ctx, next, n + 1, ncclUint8, ncclMax);
+      xbytes += 2 * (int64_t)(P - 1) * (n + 1) / P;
       INL_CUDA(cudaMemcpyAsync(ctx->pinned, next + n, 1, cudaMemcpyDeviceToHost, st));
       ctx_sync(ctx);
       if (*(volatile uint8_t *)ctx->pinned == 0) break;
@@ -1736,7 +1778,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       ++L;
     }
   }
-  finish_stats(ctx, f, stats, L, ftotal);
+  finish_stats(ctx, f, stats, L, ftotal, xbytes);
 }
 
 }  // namespace inl

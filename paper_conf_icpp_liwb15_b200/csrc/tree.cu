@@ -200,6 +200,7 @@ void tree_run(inl_ctx ctx, const inl_csr &T, const int32_t *parent, int64_t root
     stats->frontier_total = bst.frontier_total;
     stats->launches = launches;
     stats->host_syncs = bst.host_syncs + 1;
+    stats->exchange_bytes = 0;
   }
 }
 

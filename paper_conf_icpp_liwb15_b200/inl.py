@@ -51,7 +51,7 @@ class BinsT(C.Structure):
 
 class StatsT(C.Structure):
     _fields_ = [("iterations", C.c_int32), ("edges_relaxed", C.c_int64), ("frontier_total", C.c_int64),
-                ("launches", C.c_int64), ("host_syncs", C.c_int64)]
+                ("launches", C.c_int64), ("host_syncs", C.c_int64), ("exchange_bytes", C.c_int64)]
 
 
 class PlanInfoT(C.Structure):
@@ -341,7 +341,8 @@ def sssp(ctx: Ctx, G: Csr, w, source: int, dist, plan: Plan | None = None) -> di
     _check(lib().inl_sssp(ctx.handle, C.byref(s), _ptr(w), int(source), _ptr(dist), C.byref(st),
                           _plan_handle(plan)), ctx)
     return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total,
-            "launches": st.launches, "host_syncs": st.host_syncs}
+            "launches": st.launches, "host_syncs": st.host_syncs,
+            "exchange_bytes": st.exchange_bytes}
 
 
 def bfs(ctx: Ctx, G: Csr, source: int, level, plan: Plan | None = None) -> dict:
@@ -352,7 +353,8 @@ def bfs(ctx: Ctx, G: Csr, source: int, level, plan: Plan | None = None) -> dict:
     _check(lib().inl_bfs(ctx.handle, C.byref(s), int(source), _ptr(level), C.byref(st),
                          _plan_handle(plan)), ctx)
     return {"iterations": st.iterations, "edges_relaxed": st.edges_relaxed, "frontier_total": st.frontier_total,
-            "launches": st.launches, "host_syncs": st.host_syncs}
+            "launches": st.launches, "host_syncs": st.host_syncs,
+            "exchange_bytes": st.exchange_bytes}
 
 
 def bc(ctx: Ctx, G: Csr, sources, out, plan: Plan | None = None) -> dict:

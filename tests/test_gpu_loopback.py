@@ -251,3 +251,35 @@ def test_row_block_checks(g12_dir):
         inl.spmv_allgather(ctx, A, dev(np.ones(A.nnz, np.float32)), dev(np.ones(n, np.float32)), y)
     _, errs = run_ranks(2, fn, timeout=120)
     assert len(errs) == 2 and all("INVALID_ARGUMENT" in e or "NCCL" in e for _, e in errs)
+
+
+@pytest.mark.parametrize("P", [2, 8])
+def test_exchange_volume_fused_vs_collective(g18_sym, P, monkeypatch):
+    """NEXT-1's exchange volume against the r01 collectives, per rank and BFS / SSSP call
+    (inl_stats.exchange_bytes): same results, and the record lands in the test log."""
+    g, w = g18_sym
+    s = inlgen.sources(g.row_ptr, 1)[0]
+    n = g.n_global
+    b = inl.partition_rows(n, P)
+    vols = {}
+    for mode in ("fused", "collective"):
+        if mode == "collective":
+            monkeypatch.setenv("INL_BFS_EXCHANGE", "bytemap")
+            monkeypatch.setenv("INL_SSSP_EXCHANGE", "dense")
+
+        def fn(r, ctx):
+            rp, ci, wl = block(g.row_ptr, g.col_idx, b[r], b[r + 1], w)
+            A = inl.Csr(dev(rp), dev(ci), n, b[r])
+            d = torch.empty(n, dtype=torch.int32, device="cuda")
+            st_s = inl.sssp(ctx, A, dev(wl.view(np.int32)), s, d)
+            lv = torch.empty(n, dtype=torch.int32, device="cuda")
+            st_b = inl.bfs(ctx, A, s, lv)
+            return d.cpu().numpy(), lv.cpu().numpy(), st_s["exchange_bytes"], st_b["exchange_bytes"]
+        res, errs = run_ranks(P, fn)
+        assert not errs, errs
+        vols[mode] = (max(r[2] for r in res), max(r[3] for r in res))
+        assert np.array_equal(res[0][0].view(np.uint32), oracle.sssp(g.row_ptr, g.col_idx, w, s))
+        assert np.array_equal(res[0][1], oracle.bfs(g.row_ptr, g.col_idx, s))
+    print(f"\nexchange bytes per rank, scale 18, P={P}: SSSP fused {vols['fused'][0]} vs dense "
+          f"{vols['collective'][0]}; BFS fused {vols['fused'][1]} vs byte map {vols['collective'][1]}")
+    assert vols["fused"][0] > 0 and vols["fused"][1] > 0
