@@ -914,22 +914,28 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
   }
 }
 
-// warp bin, first pass: 8-lane groups, 4 vertices per warp, 16 neighbours per step (two
-// loads per lane in flight), at most kBuGroupSpan neighbours: in a bottom-up level almost every
-// high-degree vertex has a frontier neighbour among its first few (R-MAT scale 22: median
-// position 4, 90th percentile 14), so a whole warp per vertex would mostly read wasted lanes.
-// A vertex whose first kBuGroupSpan neighbours hold no parent goes to the deep list.
+// Group-mapped bottom-up scan: G lanes per vertex (32/G vertices per warp), 2G neighbours per
+// step (two loads per lane in flight, consecutive lanes on consecutive neighbours: one sector
+// serves a group's load instead of one per lane), early exit on the group's ballot, at most
+// SPAN neighbours; with DEFER a vertex whose first SPAN neighbours hold no parent goes to the
+// deep list.  Warp bin: G = 8, SPAN = 64 — in a bottom-up level almost every high-degree vertex
+// has a frontier neighbour among its first few (R-MAT scale 22: median position 4, 90th
+// percentile 14), so a whole warp per vertex would mostly read wasted lanes.  Thread bin (the
+// vertices of <= kBuThread neighbours): G = 4 covers a vertex in <= 4 steps with 4x fewer
+// L1TEX wavefronts for the column loads than one lane per vertex (`k_bu_thread`).
 constexpr int kBuGroup = 8;
 constexpr int kBuGroupSpan = 64;
 
-__global__ void __launch_bounds__(256) k_bu_warp(BuArgs a, int32_t *deep, int *n_deep) {
+template <int G, int SPAN, bool DEFER>
+__global__ void __launch_bounds__(256) k_bu_group(BuArgs a, int32_t *deep, int *n_deep) {
   a.pol = policy_evict_first();
-  const int lane = threadIdx.x & 31, gl = lane & (kBuGroup - 1), gsh = lane & ~(kBuGroup - 1);
-  const int64_t ngroups = ((int64_t)gridDim.x * blockDim.x) / kBuGroup;
-  const int64_t nn = ((int64_t)a.n_in + 3) / 4 * 4;  // a warp's 4 groups iterate together
+  const int lane = threadIdx.x & 31, gl = lane & (G - 1), gsh = lane & ~(G - 1);
+  constexpr unsigned GM = G == 32 ? 0xffffffffu : ((1u << G) - 1u);
+  const int64_t ngroups = ((int64_t)gridDim.x * blockDim.x) / G;
+  const int64_t nn = ((int64_t)a.n_in + (32 / G) - 1) / (32 / G) * (32 / G);  // a warp's groups iterate together
   int fcnt = 0;
   unsigned long long dg = 0, ex = 0;
-  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / kBuGroup; i < nn; i += ngroups) {
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G; i < nn; i += ngroups) {
     const bool valid = i < a.n_in;
     const int32_t v = valid ? a.in[i] : 0;
     int64_t s = 0, e = 0;
@@ -937,31 +943,31 @@ __global__ void __launch_bounds__(256) k_bu_warp(BuArgs a, int32_t *deep, int *n
       s = a.rp[v];
       e = a.rp[v + 1];
     }
-    const int64_t stop = min(e, s + kBuGroupSpan);
+    const int64_t stop = min(e, s + SPAN);
     bool found = false;
-    for (int64_t k = s;; k += 2 * kBuGroup) {
+    for (int64_t k = s;; k += 2 * G) {
       const bool act = k < stop && !found;
       if (!__any_sync(0xffffffffu, act)) break;
       bool hit = false;
       if (act) {
-        const int64_t k0 = k + gl, k1 = k + kBuGroup + gl;
+        const int64_t k0 = k + gl, k1 = k + G + gl;
         const int32_t u0 = k0 < stop ? (int32_t)ld_stream_pol(a.col + k0, a.pol) : -1;
         const int32_t u1 = k1 < stop ? (int32_t)ld_stream_pol(a.col + k1, a.pol) : -1;
         const uint32_t f0 = u0 >= 0 ? __ldg(a.fcur + (u0 >> 5)) : 0u;
         const uint32_t f1 = u1 >= 0 ? __ldg(a.fcur + (u1 >> 5)) : 0u;
         hit = (u0 >= 0 && ((f0 >> (u0 & 31)) & 1u)) || (u1 >= 0 && ((f1 >> (u1 & 31)) & 1u));
-        if (gl == 0) ex += (unsigned long long)min((int64_t)(2 * kBuGroup), stop - k);
+        if (gl == 0) ex += (unsigned long long)min((int64_t)(2 * G), stop - k);
       }
       const unsigned m = __ballot_sync(0xffffffffu, hit);
-      if ((m >> gsh) & ((1u << kBuGroup) - 1u)) found = true;
+      if ((m >> gsh) & GM) found = true;
     }
     if (gl == 0 && valid) {
       if (found) {
         bu_visit(a, v);
         ++fcnt;
         dg += (unsigned long long)(e - s);
-      } else if (e > stop) {
-        deep[atomicAdd(n_deep, 1)] = v;  // rare: no parent among the first kBuGroupSpan
+      } else if (DEFER && e > stop) {
+        deep[atomicAdd(n_deep, 1)] = v;  // rare: no parent among the first SPAN
       }
     }
   }
@@ -1630,6 +1636,8 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
     const char *e = getenv("INL_BFS_BU");
     bu_word = e && std::string(e) == "word";
   }
+  const char *bs_env = getenv("INL_BFS_SMALL");
+  const bool bu_small_thread = bs_env && std::string(bs_env) == "thread";
   int32_t *bl_s[2] = {nullptr, nullptr}, *bl_l[2] = {nullptr, nullptr};
   int n_small = 0, n_large = 0, bl_cur = 0;
   bool lists_ok = false;  // the worklists hold exactly the unvisited vertices of degree > 0
@@ -1684,8 +1692,14 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           INL_CUDA(cudaMemsetAsync(f.counts + 6, 0, 2 * sizeof(int), st));
           BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, f.counts, mfp, 0, f.relaxed};
           if (n_small > 0) {
-            KScope ks(ctx, "k_bu_thread");
-            k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
+            if (bu_small_thread) {  // INL_BFS_SMALL=thread: one lane per vertex (measurement switch)
+              KScope ks(ctx, "k_bu_thread");
+              k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
+            } else {
+              KScope ks(ctx, "k_bu_small");
+              k_bu_group<4, kBuThread, false><<<grid_for((int64_t)n_small * 4, ctx->num_sms), 256, 0, st>>>(ba, nullptr,
+                                                                                                   nullptr);
+            }
           }
           ba.in = bl_l[bl_cur];
           ba.n_in = n_large;
@@ -1694,7 +1708,8 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
             INL_CUDA(cudaMemsetAsync(f.counts + 3, 0, sizeof(int), st));
             {
               KScope ks(ctx, "k_bu_warp");
-              k_bu_warp<<<grid_for((int64_t)n_large * kBuGroup, ctx->num_sms), 256, 0, st>>>(ba, deep, f.counts + 3);
+              k_bu_group<kBuGroup, kBuGroupSpan, true><<<grid_for((int64_t)n_large * kBuGroup, ctx->num_sms), 256, 0, st>>>(
+                  ba, deep, f.counts + 3);
             }
             KScope ks(ctx, "k_bu_deep");
             k_bu_deep<<<ctx->num_sms * 2, 256, 0, st>>>(ba, deep, f.counts + 3);
