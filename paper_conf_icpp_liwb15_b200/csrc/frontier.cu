@@ -921,8 +921,9 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
 // deep list.  Warp bin: G = 8, SPAN = 64 — in a bottom-up level almost every high-degree vertex
 // has a frontier neighbour among its first few (R-MAT scale 22: median position 4, 90th
 // percentile 14), so a whole warp per vertex would mostly read wasted lanes.  Thread bin (the
-// vertices of <= kBuThread neighbours): G = 4 covers a vertex in <= 4 steps with 4x fewer
-// L1TEX wavefronts for the column loads than one lane per vertex (`k_bu_thread`).
+// vertices of <= kBuThread neighbours) as 4-lane groups (INL_BFS_SMALL=group): 4x fewer L1TEX
+// wavefronts for the column loads than one lane per vertex, but measured no faster (scale 26:
+// 0.47 vs 0.43 ms per launch) — the random frontier-bit probes bound it; k_bu_thread stays.
 constexpr int kBuGroup = 8;
 constexpr int kBuGroupSpan = 64;
 
@@ -1636,8 +1637,10 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
     const char *e = getenv("INL_BFS_BU");
     bu_word = e && std::string(e) == "word";
   }
+  // thread bin: one lane per vertex (default) or 4-lane groups (INL_BFS_SMALL=group: coalesced
+  // column loads, measured no faster — the frontier-bit probes, not the column loads, bound it)
   const char *bs_env = getenv("INL_BFS_SMALL");
-  const bool bu_small_thread = bs_env && std::string(bs_env) == "thread";
+  const bool bu_small_thread = !(bs_env && std::string(bs_env) == "group");
   int32_t *bl_s[2] = {nullptr, nullptr}, *bl_l[2] = {nullptr, nullptr};
   int n_small = 0, n_large = 0, bl_cur = 0;
   bool lists_ok = false;  // the worklists hold exactly the unvisited vertices of degree > 0
@@ -1692,7 +1695,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           INL_CUDA(cudaMemsetAsync(f.counts + 6, 0, 2 * sizeof(int), st));
           BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, f.counts, mfp, 0, f.relaxed};
           if (n_small > 0) {
-            if (bu_small_thread) {  // INL_BFS_SMALL=thread: one lane per vertex (measurement switch)
+            if (bu_small_thread) {
               KScope ks(ctx, "k_bu_thread");
               k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
             } else {
