@@ -165,8 +165,16 @@ inl_status inl_partition_rows(int64_t n, int32_t nranks, int64_t *bounds);
  * (torch.distributed in the Python binding); every rank then calls inl_comm_init.
  * Once a ctx has a communicator it is one rank of a row-block job: its CSR is
  * the row block [rank*B, rank*B + n_rows), B = ceil(n_global / nranks), and the ops run the
- * exchange of SURVEY §8a row a12 (PageRank allgather, SSSP allreduce-min, BFS
- * allreduce-max; inl_spmv_allgather).  nranks = 1 is allowed (the same code path). */
+ * exchange of SURVEY §8a row a12: PageRank allgathers its contributions in K row sub-blocks
+ * overlapped with the gather; SpMV allgathers y in inl_spmv_allgather; BFS and
+ * SSSP use the fused peer-memory exchange of SURVEY §8f NEXT-1 — discovered vertices set bits
+ * in their owners' next-frontier bitmaps, improved distances are atomicMin'd into their owners'
+ * arrays, over NVLink peer memory mapped with CUDA IPC (handles exchanged through NCCL), one
+ * barrier / one 4-byte allreduce per round — or, with the environment variables
+ * INL_BFS_EXCHANGE=bytemap / INL_SSSP_EXCHANGE=dense, an n-byte allreduce-max / a 4n-byte
+ * allreduce-min per round.  While waiting, NCCL ranks poll ncclCommGetAsyncError: a failed peer
+ * or a collective stuck for INL_NCCL_TIMEOUT_S seconds (default 600) aborts the communicator
+ * and the call returns INL_ERR_NCCL.  nranks = 1 is allowed (the same code path). */
 inl_status inl_nccl_unique_id(uint8_t out[128]);
 inl_status inl_comm_init(inl_ctx ctx, const uint8_t uid[128], int32_t nranks, int32_t rank);
 
@@ -219,16 +227,17 @@ inl_status inl_spmv_allgather(inl_ctx ctx, const inl_csr *A, const float *val, c
 inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_degree, float damping,
                         int32_t iterations, float *rank, inl_plan plan);
 
-/* SSSP (P5@10241, P11@2218): frontier Bellman-Ford relaxation (atomicMin) until
- * no distance changes (one GPU: near-far scheduled, the step loop as one CUDA-graph launch).  w [nnz] uint32 >= 1, dist [n_global] uint32 with
- * UINT32_MAX = unreachable (replicated).  Distances must stay < 2^32 - 2^8.
- * Blocks until converged. */
+/* SSSP (P5@10241, P11@2218): frontier Bellman-Ford relaxation (atomicMin) until no distance
+ * changes (one GPU: near-far scheduled, the step loop as one CUDA-graph launch).  w [nnz]
+ * uint32 >= 1, dist [n_global] uint32 with UINT32_MAX = unreachable (replicated).  Distances
+ * must stay < 2^32 - 2^8.  Blocks until converged. */
 inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source,
                     uint32_t *dist, inl_stats *stats, inl_plan plan);
 
-/* BFS (P5@11591): level-synchronous frontier expansion (direction-optimizing when the
- * plan found the graph symmetric); level [n_global] int32,
- * -1 = unreachable, level[source] = 0 (replicated).  Blocks until converged. */
+/* BFS (P5@11591): level-synchronous frontier expansion (one GPU: direction-optimizing when the
+ * plan found the graph symmetric, bottom-up levels over degree-binned worklists of the unvisited
+ * vertices); level [n_global] int32, -1 = unreachable, level[source] = 0 (replicated).
+ * Blocks until converged. */
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
                    inl_stats *stats, inl_plan plan);
 
