@@ -257,7 +257,7 @@ def run_inl(a):
     # the dominant kernel(s), timed live by the library with events on its own stream
     kernels = (["k_gather", "k_gather_chunks", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
                else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
-               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_level", "k_bu_thread", "k_bu_small", "k_bu_warp", "k_bu_deep",
+               else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_thread", "k_bu_small", "k_bu_warp", "k_bu_deep",
                      "k_sssp_split", "sssp_graph"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]

@@ -986,104 +986,6 @@ __global__ void __launch_bounds__(256) k_bu_group(BuArgs a, int32_t *deep, int *
   }
 }
 
-// Bottom-up level over the whole vertex range with the paper's template inside each CTA
-// (dbuf-shared, P5@3623): one thread per vertex; an unvisited vertex of degree <= kBuThread
-// scans its neighbours serially (thread-mapped, 8 loads in flight, early exit at the first
-// frontier neighbour); larger ones go to the CTA's shared buffer and are scanned by 8-lane
-// groups (16 neighbours per step over the first kBuGroupSpan), the rest to the global deep
-// list.  No worklists to build or carry: a visited vertex costs one bit of a bitmap word the
-// warp reads anyway.
-__global__ void __launch_bounds__(256) k_bu_level(BuArgs a, int64_t n, int32_t *deep, int *n_deep) {
-  __shared__ int32_t buf[256];
-  __shared__ int nb;
-  a.pol = policy_evict_first();
-  const int tid = threadIdx.x, lane = tid & 31, gl = lane & (kBuGroup - 1), gsh = lane & ~(kBuGroup - 1);
-  int fcnt = 0;
-  unsigned long long dg = 0, ex = 0;
-  for (int64_t r0 = blockIdx.x * 256LL; r0 < n; r0 += (int64_t)gridDim.x * 256) {
-    if (tid == 0) nb = 0;
-    __syncthreads();
-    const int64_t v = r0 + tid;
-    if (v < n && !((a.visited[v >> 5] >> (v & 31)) & 1u)) {
-      const int64_t s = a.rp[v], e = a.rp[v + 1];
-      if (e - s > kBuThread) {
-        buf[atomicAdd(&nb, 1)] = (int32_t)v;
-      } else if (e > s) {  // thread bin
-        bool found = false;
-        for (int64_t k = s; k < e && !found; k += 8) {
-          ex += (unsigned long long)min((int64_t)8, e - k);
-          int32_t u[8];
-#pragma unroll
-          for (int j = 0; j < 8; ++j) u[j] = k + j < e ? (int32_t)ld_stream_pol(a.col + k + j, a.pol) : -1;
-          uint32_t fw[8];
-#pragma unroll
-          for (int j = 0; j < 8; ++j) fw[j] = u[j] >= 0 ? __ldg(a.fcur + (u[j] >> 5)) : 0u;
-#pragma unroll
-          for (int j = 0; j < 8; ++j)
-            if (u[j] >= 0 && ((fw[j] >> (u[j] & 31)) & 1u)) found = true;
-        }
-        if (found) {
-          bu_visit(a, (int32_t)v);
-          ++fcnt;
-          dg += (unsigned long long)(e - s);
-        }
-      }
-    }
-    __syncthreads();
-    const int m = nb;
-    for (int b0 = 0; b0 < m; b0 += 256 / kBuGroup) {  // the buffered (warp-bin) vertices, 8 lanes each
-      const int i = b0 + tid / kBuGroup;
-      const bool valid = i < m;
-      const int32_t w = valid ? buf[i] : 0;
-      int64_t s = 0, e = 0;
-      if (valid) {
-        s = a.rp[w];
-        e = a.rp[w + 1];
-      }
-      const int64_t stop = min(e, s + kBuGroupSpan);
-      bool found = false;
-      for (int64_t k = s;; k += 2 * kBuGroup) {
-        const bool act = k < stop && !found;
-        if (!__any_sync(0xffffffffu, act)) break;
-        bool hit = false;
-        if (act) {
-          const int64_t k0 = k + gl, k1 = k + kBuGroup + gl;
-          const int32_t u0 = k0 < stop ? (int32_t)ld_stream_pol(a.col + k0, a.pol) : -1;
-          const int32_t u1 = k1 < stop ? (int32_t)ld_stream_pol(a.col + k1, a.pol) : -1;
-          const uint32_t f0 = u0 >= 0 ? __ldg(a.fcur + (u0 >> 5)) : 0u;
-          const uint32_t f1 = u1 >= 0 ? __ldg(a.fcur + (u1 >> 5)) : 0u;
-          hit = (u0 >= 0 && ((f0 >> (u0 & 31)) & 1u)) || (u1 >= 0 && ((f1 >> (u1 & 31)) & 1u));
-          if (gl == 0) ex += (unsigned long long)min((int64_t)(2 * kBuGroup), stop - k);
-        }
-        const unsigned mk = __ballot_sync(0xffffffffu, hit);
-        if ((mk >> gsh) & 0xFFu) found = true;
-      }
-      if (gl == 0 && valid) {
-        if (found) {
-          bu_visit(a, w);
-          ++fcnt;
-          dg += (unsigned long long)(e - s);
-        } else if (e > stop) {
-          deep[atomicAdd(n_deep, 1)] = w;  // rare: no parent among the first kBuGroupSpan
-        }
-      }
-    }
-    __syncthreads();  // the buffer is reused by the next round
-  }
-  for (int o = 16; o > 0; o >>= 1) {
-    fcnt += __shfl_xor_sync(0xffffffffu, fcnt, o);
-    dg += __shfl_xor_sync(0xffffffffu, dg, o);
-    ex += __shfl_xor_sync(0xffffffffu, ex, o);
-  }
-  if (lane == 0) {
-    if (fcnt) {
-      atomicAdd(a.found, fcnt);
-      atomicAdd(a.mf, dg);
-    }
-    if (ex) atomicAdd(a.examined, ex);
-  }
-}
-
 // warp bin, deep pass: one warp per deferred vertex from neighbour kBuGroupSpan on, 64 per step,
 // early exit on __any_sync.  The count is read on the device (no host round trip).
 __global__ void __launch_bounds__(256) k_bu_deep(BuArgs a, const int32_t *deep, const int *n_deep) {
@@ -1739,16 +1641,13 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   // column loads, measured no faster — the frontier-bit probes, not the column loads, bound it)
   const char *bs_env = getenv("INL_BFS_SMALL");
   const bool bu_small_thread = !(bs_env && std::string(bs_env) == "group");
-  // default: k_bu_level (one pass over the vertex range); INL_BFS_BU=lists keeps the worklist
-  // version (CUB partition / select), =word the r01 kernel
-  const bool bu_range = !bu_word && !(getenv("INL_BFS_BU") && std::string(getenv("INL_BFS_BU")) == "lists");
   int32_t *bl_s[2] = {nullptr, nullptr}, *bl_l[2] = {nullptr, nullptr};
   int n_small = 0, n_large = 0, bl_cur = 0;
   bool lists_ok = false;  // the worklists hold exactly the unvisited vertices of degree > 0
   if (allow_bu) {
     fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
     fb = fa + nwords + 1;
-    if (!bu_word && !bu_range) {
+    if (!bu_word) {
       int32_t *L4 = (int32_t *)ctx->s_bu.get(sizeof(int32_t) * 4 * (size_t)(n + 1));
       for (int q = 0; q < 2; ++q) {
         bl_s[q] = L4 + (size_t)q * (n + 1);
@@ -1770,22 +1669,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
         }
         INL_CUDA(cudaMemsetAsync(f.counts, 0, sizeof(int), st));
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
-        if (bu_range) {  // one pass over the vertex range, binned inside each CTA
-          INL_CUDA(cudaMemsetAsync(fb, 0, sizeof(uint32_t) * nwords, st));
-          INL_CUDA(cudaMemsetAsync(f.counts + 3, 0, sizeof(int), st));
-          int32_t *deep = (int32_t *)ctx->s_bu.get(sizeof(int32_t) * (size_t)(n + 1));
-          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, nullptr, 0, f.counts, mfp, 0, f.relaxed};
-          {
-            KScope ks(ctx, "k_bu_level");
-            k_bu_level<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(ba, n, deep, f.counts + 3);
-          }
-          {
-            KScope ks(ctx, "k_bu_deep");
-            k_bu_deep<<<ctx->num_sms * 2, 256, 0, st>>>(ba, deep, f.counts + 3);
-          }
-          INL_CUDA(cudaGetLastError());
-          read_level(&nF, &mf_next);
-        } else if (bu_word) {
+        if (bu_word) {
           KScope ks(ctx, "k_bfs_bottom_up");
           k_bfs_bottom_up<<<ctx->num_sms * 8, 256, 0, st>>>(G.row_ptr, G.col_idx, n, bm, fa, fb, level, L,
                                                            f.counts, mfp);
