@@ -403,7 +403,7 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
   const int i = blockIdx.x * NT + tid;
   unsigned long long mydeg = 0;
   if (i < a.nF) {
-    const int32_t u = __ldcg(a.F + i);  // written by other CTAs (a persistent loop: not in L1)
+    const int32_t u = a.F[i];
     const int64_t rs = a.rp[u], re = a.rp[u + 1];
     const int64_t d = re - rs;
     mydeg = (unsigned long long)d;
@@ -479,7 +479,7 @@ __device__ __forceinline__ void expand_flat_dev(ExpandArgs a, Op op) {
   int64_t rs = 0;
   uint32_t su = 0;
   if (i < a.nF) {
-    const int32_t u = __ldcg(a.F + i);  // written by other CTAs (a persistent loop: not in L1)
+    const int32_t u = a.F[i];
     if (inq_prev) inq_prev[u >> 5] = 0u;  // its claim bit of the previous iteration
     rs = a.rp[u];
     const int64_t dd = a.rp[u + 1] - rs;
@@ -576,7 +576,7 @@ __device__ __forceinline__ void expand_grid_dev(ExpandArgs a, Op op) {
   __syncthreads();
   const int n = n_s;
   for (int it = blockIdx.x; it < n; it += gridDim.x) {
-    const int2 g = __ldcg(a.gitems + it);  // written by other CTAs in this step
+    const int2 g = a.gitems[it];
     const int64_t rs = a.rp[g.x], re = a.rp[g.x + 1];
     const int64_t ks = rs + (int64_t)g.y * a.chunk;
     const int64_t ke = min(ks + (int64_t)a.chunk, re);
@@ -627,7 +627,7 @@ __global__ void k_far_split(const int32_t *__restrict__ far, int nfar, const uin
                             uint32_t lo, uint32_t hi, uint32_t *inq, uint32_t *keep, int32_t *q, int *qcnt,
                             int32_t *far2, int *far2cnt) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nfar; i += gridDim.x * blockDim.x) {
-    const int32_t v = __ldcg(far + i);  // written by other CTAs
+    const int32_t v = far[i];
     const uint32_t d = dist[v];
     const uint32_t bit = 1u << (v & 31);
     if (d >= lo && d < hi) {
@@ -655,7 +655,7 @@ __device__ __forceinline__ void sssp_split_dev(SsspDyn dy, const uint32_t *__res
   const int fpar = s->fpar, par = s->par;
   const int32_t *far = dy.far[fpar];
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nfar; i += gridDim.x * blockDim.x) {
-    const int32_t v = __ldcg(far + i);  // written by other CTAs
+    const int32_t v = far[i];
     const uint32_t d = dist[v];
     if (d >= hi) {
       push(dy.far[fpar ^ 1], &dy.s->nfar2, v);
@@ -674,7 +674,7 @@ __global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) { ss
 // instead of letting a bug spin the GPU.
 constexpr int kSsspMaxSteps = 1 << 20;
 __device__ __forceinline__ void sssp_post_dev(SsspDyn dy) {
-  volatile SsspDev *s = dy.s;  // counters updated by other CTAs' atomics: read through to L2
+  SsspDev *s = dy.s;
   if (!s->done && ++s->pad > kSsspMaxSteps) s->done = 2;
   if (s->done) return;
   const bool split = s->nF == 0;
