@@ -258,7 +258,7 @@ def run_inl(a):
     kernels = (["k_gather", "k_gather_chunks", "k_cb", "k_cb_combine"] if a.op in ("spmv", "pagerank")
                else ["k_bc_fwd", "k_bc_bwd"] if a.op == "bc"
                else ["k_expand_flat", "k_expand_grid", "k_bfs_bottom_up", "k_bu_thread", "k_bu_small", "k_bu_warp", "k_bu_deep",
-                     "k_sssp_split", "sssp_graph", "sssp_persistent"])
+                     "k_sssp_split", "sssp_graph"])
     if a.thread_only:
         kernels = ["k_gather_thread_only"] if a.op == "spmv" else ["k_expand", "k_expand_grid"]
     ctx.ktimer_enable(True)

@@ -452,7 +452,7 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
 constexpr int kEdgesPerThread = 8;
 
 template <class Op>
-__device__ __forceinline__ void expand_flat_dev(ExpandArgs a, Op op) {
+__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
@@ -559,15 +559,10 @@ __device__ __forceinline__ void expand_flat_dev(ExpandArgs a, Op op) {
   op.fence();
 }
 
-template <class Op>
-__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs a, Op op) {
-  expand_flat_dev<Op>(a, op);
-}
-
 // Grid bin (dbuf-global, P5@2721): pieces of grid_chunk edges of the large-degree
 // frontier vertices, one CTA per piece (grid-stride); each thread keeps 8 edges in flight.
 template <class Op>
-__device__ __forceinline__ void expand_grid_dev(ExpandArgs a, Op op) {
+__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_grid(ExpandArgs a, Op op) {
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
@@ -598,11 +593,6 @@ __device__ __forceinline__ void expand_grid_dev(ExpandArgs a, Op op) {
     }
   }
   op.fence();
-}
-
-template <class Op>
-__global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_grid(ExpandArgs a, Op op) {
-  expand_grid_dev<Op>(a, op);
 }
 
 __global__ void k_init_sssp(uint32_t *dist, int64_t n, int64_t s) {
@@ -641,7 +631,7 @@ __global__ void k_far_split(const int32_t *__restrict__ far, int nfar, const uin
 // Device-driven step, part 1: when the near frontier is empty, advance the threshold and
 // split the far pile (duplicate-free): lo <= dist < hi -> frontier, dist >= hi -> the other
 // far buffer (stays marked in `keep`), dist < lo -> settled earlier, dropped.
-__device__ __forceinline__ void sssp_split_dev(SsspDyn dy, const uint32_t *__restrict__ dist) {
+__global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) {
   __shared__ __align__(16) SsspDev st_s;
   load_state(dy.s, &st_s);
   const SsspDev *s = &st_s;
@@ -666,16 +656,15 @@ __device__ __forceinline__ void sssp_split_dev(SsspDyn dy, const uint32_t *__res
   }
 }
 
-__global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) { sssp_split_dev(dy, dist); }
-
 // Device-driven step, part 4: roll the state over to the next step.  In the CUDA-graph loop
 // (a conditional WHILE node around the four kernels) it also sets the loop condition; a step
 // count far beyond any converging run (kSsspMaxSteps) stops the loop with an error flag
 // instead of letting a bug spin the GPU.
 constexpr int kSsspMaxSteps = 1 << 20;
-__device__ __forceinline__ void sssp_post_dev(SsspDyn dy) {
+__global__ void k_sssp_post(SsspDyn dy, cudaGraphConditionalHandle cond, int use_cond) {
   SsspDev *s = dy.s;
   if (!s->done && ++s->pad > kSsspMaxSteps) s->done = 2;
+  if (use_cond) cudaGraphSetConditional(cond, s->done ? 0u : 1u);
   if (s->done) return;
   const bool split = s->nF == 0;
   if (split) {
@@ -695,31 +684,6 @@ __device__ __forceinline__ void sssp_post_dev(SsspDyn dy) {
   s->cnt = 0;
   s->gcount = 0;
   s->slice = 0;
-}
-
-__global__ void k_sssp_post(SsspDyn dy, cudaGraphConditionalHandle cond, int use_cond) {
-  sssp_post_dev(dy);
-  if (use_cond) cudaGraphSetConditional(cond, dy.s->done ? 0u : 1u);
-}
-
-// One GPU, near-far, PERSISTENT: the whole step loop in one cooperative kernel; the four
-// phases of a step (split, flat expansion, grid pieces, roll-over) are separated by grid-wide
-// barriers instead of kernel boundaries (a step's fixed cost in the graph loop is ~45 us of
-// launches, measured by the delta sweep in profiles/r02/sssp_loops.txt).
-__global__ void __launch_bounds__(NT, 3) k_sssp_persistent(SsspDyn dy, const uint32_t *__restrict__ dist,
-                                                          ExpandArgs a, SsspOp op) {
-  cg::grid_group grid = cg::this_grid();
-  for (;;) {
-    sssp_split_dev(dy, dist);
-    grid.sync();
-    expand_flat_dev<SsspOp>(a, op);
-    grid.sync();
-    expand_grid_dev<SsspOp>(a, op);
-    grid.sync();
-    if (blockIdx.x == 0 && threadIdx.x == 0) sssp_post_dev(dy);
-    grid.sync();
-    if (*(volatile int *)&dy.s->done) break;
-  }
 }
 
 // P > 1: vertices of the owned slice whose distance dropped -> next frontier.
@@ -1317,7 +1281,7 @@ struct SsspGraph {
 void sssp_graph_free(void *g) { delete static_cast<SsspGraph *>(g); }
 
 static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, int64_t source,
-                           uint32_t *dist, inl_stats *stats, bool persistent) {
+                           uint32_t *dist, inl_stats *stats) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   FrontierBufs f = frontier_bufs(ctx, G, b);
@@ -1354,18 +1318,6 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     gm_read = true;
     if (const char *e = getenv("INL_SSSP_GRIDS")) sscanf(e, "%d,%d,%d", &gm[0], &gm[1], &gm[2]);
   }
-  if (persistent) {  // one cooperative launch: every CTA resident (the grid barriers need it)
-    static int per_sm[kMaxDevices] = {};
-    int &nb = per_sm[ctx->device % kMaxDevices];
-    if (!nb) INL_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_sssp_persistent, NT, 0));
-    INL_CHECK(nb > 0, "sssp: the persistent kernel does not fit an SM");
-    const int grid = nb * ctx->num_sms;
-    void *args[] = {&dy, &dist, &a, &op};
-    {
-      KScope ks(ctx, "sssp_persistent");
-      INL_CUDA(cudaLaunchCooperativeKernel((void *)k_sssp_persistent, grid, NT, args, 0, st));
-    }
-  } else {
   SsspGraphKey key{};
   key.rp = G.row_ptr;
   key.col = G.col_idx;
@@ -1424,7 +1376,6 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     KScope ks(ctx, "sssp_graph");
     INL_CUDA(cudaGraphLaunch(sg->exec, st));
   }
-  }
   SsspDev *hs = (SsspDev *)ctx->pinned;
   INL_CUDA(cudaMemcpyAsync(hs, dy.s, sizeof(SsspDev), cudaMemcpyDeviceToHost, st));
   ctx_sync(ctx);
@@ -1438,7 +1389,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     stats->iterations = hs->iter;
     stats->edges_relaxed = (int64_t)r;
     stats->frontier_total = (int64_t)hs->ftotal;
-    stats->launches = persistent ? 2 : 1 + 4LL * hs->pad;  // init + 4 kernels per step (one graph launch)
+    stats->launches = 1 + 4LL * hs->pad;  // init + 4 kernels per step (one graph launch)
     stats->host_syncs = 1;
     stats->exchange_bytes = 0;
   }
@@ -1459,9 +1410,8 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   const bool dyn_loop = lp && std::string(lp) == "dyn";
   if (!DIST && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && !host_loop && sssp_delta() != 0xFFFFFFFFu &&
       n > 0) {
-    const bool persistent = lp && std::string(lp) == "persistent";
     if (dyn_loop) sssp_run_dyn(ctx, G, b, w, source, dist, stats);
-    else sssp_run_graph(ctx, G, b, w, source, dist, stats, persistent);
+    else sssp_run_graph(ctx, G, b, w, source, dist, stats);
     return;
   }
   FrontierBufs f = frontier_bufs(ctx, G, b);
