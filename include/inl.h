@@ -98,9 +98,10 @@ enum {
   /* The paper's templates, as it describes them (template study):
    * lbTHRES = t_thread (rows / vertices of degree > t_thread are block-mapped).
    * SpMV: dual-queue (Fig. 1(b), P5@2074), dbuf-global and dbuf-shared (Fig. 1(c),
-   * P5@2717), CTA = cta_threads.  SSSP / BFS: dbuf-shared and dbuf-global (256-thread
-   * CTAs; plain frontier Bellman-Ford / top-down BFS like the T1 baseline).  PageRank:
-   * none (INL_ERR_UNSUPPORTED). */
+   * P5@2717), CTA = cta_threads.  SSSP / BFS: dual-queue (a pre-pass splits the frontier;
+   * thread- and block-mapped kernels), dbuf-shared and dbuf-global (256-thread CTAs; plain
+   * frontier Bellman-Ford / top-down BFS like the T1 baseline).  PageRank: none
+   * (INL_ERR_UNSUPPORTED). */
   INL_BINS_TPL_DUAL_QUEUE = 8,
   INL_BINS_TPL_DBUF_GLOBAL = 16,
   INL_BINS_TPL_DBUF_SHARED = 32

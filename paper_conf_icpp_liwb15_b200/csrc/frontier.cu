@@ -375,6 +375,56 @@ __device__ __forceinline__ bool dyn_bind<SsspOp>(ExpandArgs &a, SsspOp &op, uint
   return true;
 }
 
+// ---- the paper's dual-queue template on the frontier (Fig. 1(b), P5@2074): a pre-pass
+// "divides the elements processed in the outer loop in two queues depending on the number of
+// iterations they require in the inner-loop and processes those queues separately using thread-
+// and block-based mapping" — k_dq_split, then k_dq_thread over the small queue (one thread per
+// vertex, serial inner loop) and k_dq_block over the large one (one CTA per vertex).  Queue
+// sizes are read on the device (no host round trip).
+__global__ void k_dq_split(const int32_t *__restrict__ F, int nF, const int64_t *__restrict__ rp, int lbt,
+                           int32_t *qs, int *ns, int32_t *ql, int *nl, unsigned long long *relaxed) {
+  unsigned long long dsum = 0;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nF; i += gridDim.x * blockDim.x) {
+    const int32_t u = F[i];
+    const int64_t d = rp[u + 1] - rp[u];
+    dsum += (unsigned long long)d;
+    if (d <= lbt) push(qs, ns, u);
+    else push(ql, nl, u);
+  }
+  for (int o = 16; o > 0; o >>= 1) dsum += __shfl_xor_sync(0xffffffffu, dsum, o);
+  if ((threadIdx.x & 31) == 0 && dsum) atomicAdd(relaxed, dsum);
+}
+
+template <class Op>
+__global__ void __launch_bounds__(NT) k_dq_thread(const int32_t *__restrict__ q, const int *__restrict__ nq,
+                                                  const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                                                  Op op, int32_t *Fout, int *fcount) {
+  op.pol_stream = policy_evict_first();
+  const int n = __ldcg(nq);
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t u = q[i];
+    const uint32_t su = op.load(u);
+    for (int64_t k = rp[u]; k < rp[u + 1]; ++k) op.edge(su, k, __ldg(col + k), Fout, fcount);
+  }
+  op.fence();
+}
+
+template <class Op>
+__global__ void __launch_bounds__(NT) k_dq_block(const int32_t *__restrict__ q, const int *__restrict__ nq,
+                                                 const int64_t *__restrict__ rp, const int32_t *__restrict__ col,
+                                                 Op op, int32_t *Fout, int *fcount) {
+  op.pol_stream = policy_evict_first();
+  __shared__ int n_s;
+  if (threadIdx.x == 0) n_s = __ldcg(nq);
+  __syncthreads();
+  for (int j = blockIdx.x; j < n_s; j += gridDim.x) {
+    const int32_t u = q[j];
+    const uint32_t su = op.load(u);
+    for (int64_t k = rp[u] + threadIdx.x; k < rp[u + 1]; k += NT) op.edge(su, k, __ldg(col + k), Fout, fcount);
+  }
+  op.fence();
+}
+
 // Append the ceil(d / chunk) pieces of frontier vertex u to the grid buffer.  The buffer
 // holds gcap pieces, an upper bound of one expansion's output (frontier_cfg); a write past
 // it is dropped and flagged instead (the host turns the flag into INL_ERR_INTERNAL).
@@ -1087,10 +1137,11 @@ struct ExpandCfg {
 ExpandCfg expand_cfg(const inl_csr &G, const Bins &b) {
   ExpandCfg c{b.t_thread, b.t_warp, b.t_block, std::min(b.grid_chunk, 2048), true, 0};
   const int tpl = b.flags & kTemplateFlags;
-  INL_CHECK(tpl != INL_BINS_TPL_DUAL_QUEUE, "dual-queue template: SpMV only (SSSP/BFS: dbuf-shared, dbuf-global)");
-  if (tpl) {  // the paper's delayed-buffer templates (template study): lbTHRES = t_thread
+  if (tpl) {  // the paper's templates (template study): lbTHRES = t_thread
     c.t_warp = b.t_thread;  // no warp bin: above lbTHRES is block-mapped ...
-    c.t_block = tpl == INL_BINS_TPL_DBUF_SHARED ? INT32_MAX / 2 : b.t_thread;  // ... in smem / via the grid buffer
+    // ... in smem (dbuf-shared), via the grid buffer (dbuf-global), or from the large queue of
+    // the pre-pass (dual-queue: no grid buffer)
+    c.t_block = tpl == INL_BINS_TPL_DBUF_GLOBAL ? b.t_thread : INT32_MAX / 2;
   }
   c.flat = !((b.flags & INL_BINS_THREAD_ONLY) || tpl);
   const int64_t T = c.flat ? c.t_warp : c.t_block;
@@ -1128,6 +1179,27 @@ void expand(inl_ctx ctx, const inl_csr &G, const Bins &b, FrontierBufs &f, int n
   const ExpandCfg c = expand_cfg(G, b);
   ExpandArgs a{f.F, nF, G.row_ptr, G.col_idx, c.t_thread, c.t_warp, c.t_block, c.chunk,
                f.gitems, f.counts + 1, (int)f.gcap, f.counts + 2, f.Fout, f.counts, f.relaxed};
+  if ((b.flags & kTemplateFlags) == INL_BINS_TPL_DUAL_QUEUE) {
+    int32_t *qs = (int32_t *)ctx->s_bu.get(sizeof(int32_t) * 2 * (size_t)(G.n_rows + 1));
+    int32_t *ql = qs + G.n_rows + 1;
+    INL_CUDA(cudaMemsetAsync(f.counts + 4, 0, 2 * sizeof(int), st));
+    if (nF > 0) {
+      {
+        KScope ks(ctx, "k_dq_split");
+        k_dq_split<<<grid_for(nF, ctx->num_sms), NT, 0, st>>>(f.F, nF, G.row_ptr, c.t_thread, qs, f.counts + 4, ql,
+                                                             f.counts + 5, f.relaxed);
+      }
+      {
+        KScope ks(ctx, "k_dq_thread");
+        k_dq_thread<Op><<<grid_for(nF, ctx->num_sms), NT, 0, st>>>(qs, f.counts + 4, G.row_ptr, G.col_idx, op, f.Fout,
+                                                                  f.counts);
+      }
+      KScope ks(ctx, "k_dq_block");
+      k_dq_block<Op><<<ctx->num_sms * 8, NT, 0, st>>>(ql, f.counts + 5, G.row_ptr, G.col_idx, op, f.Fout, f.counts);
+    }
+    INL_CUDA(cudaGetLastError());
+    return;
+  }
   if (nF > 0) {
     if (!c.flat) {  // the paper's baseline (thread-mapped) / templates
       KScope ks(ctx, "k_expand");

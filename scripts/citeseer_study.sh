@@ -5,7 +5,7 @@ mkdir -p gpurun_out
 M=gpu__time_duration.sum,smsp__thread_inst_executed_per_inst_executed.ratio,smsp__sass_average_data_bytes_per_sector_mem_global_op_ld.pct,smsp__sass_average_data_bytes_per_sector_mem_global_op_st.pct
 timeout 900 python scripts/template_study.py --graph citeseer > gpurun_out/ts_spmv_citeseer.jsonl 2> gpurun_out/ts_spmv_citeseer.err
 timeout 900 python scripts/template_study_sssp.py --graph citeseer --sources 3 > gpurun_out/ts_sssp_citeseer.jsonl 2> gpurun_out/ts_sssp_citeseer.err
-for v in thread_only dbuf_shared:32 dbuf_shared:64 dbuf_shared:256 dbuf_shared:1024 dbuf_global:32 dbuf_global:128 default; do
+for v in thread_only dual_queue:32 dbuf_shared:32 dbuf_shared:64 dbuf_shared:256 dbuf_shared:1024 dbuf_global:32 dbuf_global:128 default; do
   f=$(echo $v | tr ':' '_')
   timeout 600 ncu --metrics $M --clock-control none --csv --log-file gpurun_out/eff_sssp_$f.csv python scripts/template_study_sssp.py --graph citeseer --sources 1 --only $v > /dev/null 2>&1
 done

@@ -63,7 +63,8 @@ def main():
     d = torch.empty(A.n_global, dtype=torch.int32, device="cuda")
     ref = {}
     variants = [("thread_only (T1)", dict(flags=inl.BINS_THREAD_ONLY), None)]
-    for name, fl in (("dbuf_shared", inl.BINS_TPL_DBUF_SHARED), ("dbuf_global", inl.BINS_TPL_DBUF_GLOBAL)):
+    for name, fl in (("dual_queue", inl.BINS_TPL_DUAL_QUEUE), ("dbuf_shared", inl.BINS_TPL_DBUF_SHARED),
+                     ("dbuf_global", inl.BINS_TPL_DBUF_GLOBAL)):
         for lbt in (32, 64, 128, 256, 1024):
             variants.append((name, dict(t_thread=lbt, t_warp=max(lbt, 16), t_block=max(lbt, 16), flags=fl), lbt))
     variants.append(("default (flat + grid, near-far)", dict(), None))

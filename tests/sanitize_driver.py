@@ -39,7 +39,7 @@ def main():
     ps = inl.Plan(ctx, As)  # symmetric plan: BFS bottom-up steps, BC pull steps
     inl.bfs(ctx, As, src, d, ps)
     inl.sssp(ctx, As, w, src, d, inl.Plan(ctx, As, inl.bins(flags=inl.BINS_SSSP_DEVLOOP)))
-    for fl in (inl.BINS_TPL_DBUF_SHARED, inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_THREAD_ONLY):
+    for fl in (inl.BINS_TPL_DBUF_SHARED, inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DUAL_QUEUE, inl.BINS_THREAD_ONLY):
         pt = inl.Plan(ctx, As, inl.bins(t_thread=16, t_warp=16, t_block=16, flags=fl))
         inl.sssp(ctx, As, w, src, d, pt)
         inl.bfs(ctx, As, src, d, pt)

@@ -82,10 +82,10 @@ def test_template_flags_are_spmv_only(ctx, g14):
             inl.Plan(ctx, A, inl.bins(flags=fl))
 
 
-@pytest.mark.parametrize("name", ["dbuf_global", "dbuf_shared"])
+@pytest.mark.parametrize("name", ["dbuf_global", "dbuf_shared", "dual_queue"])
 @pytest.mark.parametrize("lbt", [0, 8, 32, 1024])
 def test_frontier_templates_bit_exact(ctx, name, lbt):
-    """SSSP / BFS through the paper's delayed-buffer templates (plain frontier Bellman-Ford)."""
+    """SSSP / BFS through the paper's templates (plain frontier Bellman-Ford / top-down BFS)."""
     g = inlgen.host_build(12, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
     w = inlgen.weights_host(g.row_ptr, g.col_idx)
     A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
@@ -100,9 +100,23 @@ def test_frontier_templates_bit_exact(ctx, name, lbt):
         assert np.array_equal(lv.cpu().numpy(), oracle.bfs(g.row_ptr, g.col_idx, s))
 
 
-def test_dual_queue_is_spmv_only_for_frontiers(ctx):
-    g = inlgen.host_build(10, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
-    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
-    lv = torch.zeros(g.n_global, dtype=torch.int32, device="cuda")
-    with pytest.raises(RuntimeError):
-        inl.bfs(ctx, A, 0, lv, inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DUAL_QUEUE)))
+def test_dual_queue_frontier_hub_and_empty(ctx):
+    """Dual-queue on the frontier: a hub far above lbTHRES (large queue, one CTA) next to a path,
+    and an isolated source (empty queues)."""
+    n = 30000
+    e = [(0, i) for i in range(1, n - 100)] + [(i, i + 1) for i in range(n - 101, n - 1)]
+    rp, ci, w = csr_from_edges(n, e, np.arange(len(e)) % 255 + 1, symmetric=True)
+    A = inl.Csr(dev(rp), dev(ci), n)
+    plan = inl.Plan(ctx, A, inl.bins(t_thread=32, flags=inl.BINS_TPL_DUAL_QUEUE))
+    for s in (0, n - 1, 5):
+        d = torch.zeros(n, dtype=torch.int32, device="cuda")
+        inl.sssp(ctx, A, dev(w.view(np.int32)), s, d, plan)
+        assert np.array_equal(d.cpu().numpy().view(np.uint32), oracle.sssp(rp, ci, w, s))
+        lv = torch.zeros(n, dtype=torch.int32, device="cuda")
+        inl.bfs(ctx, A, s, lv, plan)
+        assert np.array_equal(lv.cpu().numpy(), oracle.bfs(rp, ci, s))
+    rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3)], [5, 6], symmetric=True)
+    A = inl.Csr(dev(rp), dev(ci), 6)
+    d = torch.zeros(6, dtype=torch.int32, device="cuda")
+    inl.sssp(ctx, A, dev(w.view(np.int32)), 0, d, inl.Plan(ctx, A, inl.bins(t_thread=1, flags=inl.BINS_TPL_DUAL_QUEUE)))
+    assert d.cpu().numpy().view(np.uint32).tolist() == [0] + [0xFFFFFFFF] * 5
