@@ -100,8 +100,9 @@ enum {
    * SpMV: dual-queue (Fig. 1(b), P5@2074), dbuf-global and dbuf-shared (Fig. 1(c),
    * P5@2717), CTA = cta_threads.  SSSP / BFS: dual-queue (a pre-pass splits the frontier;
    * thread- and block-mapped kernels), dbuf-shared and dbuf-global (256-thread CTAs; plain
-   * frontier Bellman-Ford / top-down BFS like the T1 baseline).  PageRank: none
-   * (INL_ERR_UNSUPPORTED). */
+   * frontier Bellman-Ford / top-down BFS like the T1 baseline).  PageRank (one GPU): each
+   * iteration is the template SpMV with unit values over the in-CSR, then an elementwise
+   * update (INL_BINS_THREAD_ONLY: the T1 gather). */
   INL_BINS_TPL_DUAL_QUEUE = 8,
   INL_BINS_TPL_DBUF_GLOBAL = 16,
   INL_BINS_TPL_DBUF_SHARED = 32

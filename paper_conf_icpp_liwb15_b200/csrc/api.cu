@@ -700,11 +700,12 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
     inl_csr d = device_csr(ctx, A_in);
     const int32_t *dod = stage_in(ctx, ctx->h_od, out_degree, A_in->n_global);
     StagedOut<float> ro = stage_out(ctx->h_y, rank, A_in->n_global);
-    if (plan && (plan->bins.flags & INL_BINS_THREAD_ONLY))
-      raise(INL_ERR_UNSUPPORTED, "thread-only baseline plans are SpMV/SSSP/BFS only");
-    if (plan && (plan->bins.flags & kTemplateFlags))
-      raise(INL_ERR_UNSUPPORTED, "paper-template plans (INL_BINS_TPL_*) are SpMV only");
-    pagerank_run(ctx, get_plan(ctx, d, plan), dod, damping, iterations, ro.dev);
+    if (plan && (plan->bins.flags & (kTemplateFlags | INL_BINS_THREAD_ONLY))) {  // the template study (one GPU)
+      INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
+      pagerank_run(ctx, plan, dod, damping, iterations, ro.dev);
+    } else {
+      pagerank_run(ctx, get_plan(ctx, d, plan), dod, damping, iterations, ro.dev);
+    }
     finish_out(ctx, ro);
   });
 }

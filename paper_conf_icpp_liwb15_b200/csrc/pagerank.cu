@@ -153,6 +153,47 @@ __global__ void k_remap_hot(const int32_t *__restrict__ hot, int n_hot, const in
   }
 }
 
+// Template-study PageRank (the paper's Fig. 6 / Table II PageRank rows): contributions in vertex
+// space; c[v] = PR^0/outdeg for v with out-links, 0 otherwise; dangling count for D^0.
+__global__ void k_pr_init_v(const int32_t *__restrict__ od, int64_t n, float *__restrict__ c,
+                            unsigned long long *__restrict__ n_dangling) {
+  const float pr0 = (float)(1.0 / (double)n);
+  unsigned long long cnt = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const int d = od[v];
+    c[v] = d > 0 ? pr0 / (float)d : 0.0f;
+    cnt += d == 0;
+  }
+  for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(n_dangling, cnt);
+}
+
+// PR'(v) = base + d * s(v); the next contribution in place of c (the gather that read c is
+// done); the rank on the last step; one fixed-order fp64 dangling partial per CTA
+__global__ void __launch_bounds__(256) k_pr_apply_v(const float *__restrict__ s, const int32_t *__restrict__ od,
+                                                    const float *__restrict__ base_p, float damping, int64_t n,
+                                                    float *__restrict__ c, float *__restrict__ rank_out,
+                                                    double *__restrict__ dpart) {
+  __shared__ double red[8];
+  const float base = *base_p;
+  double dsum = 0.0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const float pr = fmaf(damping, s[v], base);
+    const int d = od[v];
+    c[v] = d > 0 ? pr / (float)d : 0.0f;
+    if (rank_out) rank_out[v] = pr;
+    if (d == 0) dsum += (double)pr;
+  }
+  for (int o = 16; o > 0; o >>= 1) dsum += __shfl_xor_sync(0xffffffffu, dsum, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = dsum;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int q = 0; q < 8; ++q) t += red[q];
+    dpart[blockIdx.x] = t;
+  }
+}
+
 int grid_for(int64_t n, int sms) {
   int64_t g = (n + 255) / 256;
   if (g > (int64_t)sms * 16) g = (int64_t)sms * 16;
@@ -280,8 +321,53 @@ static int pr_subblocks() {
   return k < 1 ? 1 : k > 16 ? 16 : k;
 }
 
+// PageRank through the paper's templates (INL_BINS_TPL_*) or its thread-mapped baseline T1
+// (INL_BINS_THREAD_ONLY), one GPU, for the template study: per
+// iteration the template SpMV with implicit unit values gathers s(v) = sum of c(u) over the
+// in-CSR, then k_pr_apply_v forms PR', the next contributions and the dangling partials.
+static void pagerank_template(inl_ctx ctx, inl_plan p, const int32_t *od, float damping, int iters, float *rank) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = p->n_global;
+  inl_csr A{p->n_rows, p->n_global, p->row_begin, p->nnz, p->row_ptr, p->col_idx};
+  float *c = (float *)ctx->s_a.get(sizeof(float) * (size_t)n);
+  float *s = (float *)ctx->s_b.get(sizeof(float) * (size_t)n);
+  const int grid = grid_for(n, ctx->num_sms);
+  char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (size_t)grid);
+  float *base = (float *)scal;
+  unsigned long long *ndang = (unsigned long long *)(scal + 8);
+  double *dall = (double *)(scal + 16);
+  double *dpart = (double *)(scal + 256);
+  INL_CUDA(cudaMemsetAsync(ndang, 0, sizeof(unsigned long long), st));
+  k_pr_init_v<<<grid, 256, 0, st>>>(od, n, c, ndang);
+  k_pr_base0<<<1, 1, 0, st>>>(ndang, n, (double)damping, base);
+  INL_CUDA(cudaGetLastError());
+  for (int t = 0; t < iters; ++t) {
+    const bool last = t + 1 == iters;
+    if (p->bins.flags & INL_BINS_THREAD_ONLY) spmv_thread_only(ctx, A, nullptr, c, s);  // the T1 baseline
+    else spmv_template(ctx, A, p->bins, nullptr, c, s);
+    k_pr_apply_v<<<grid, 256, 0, st>>>(s, od, base, damping, n, c, last ? rank : nullptr, dpart);
+    if (!last) {
+      k_pr_dsum<<<1, 1024, 0, st>>>(dpart, grid, dall);
+      k_pr_base<<<1, 1, 0, st>>>(dall, 1, n, (double)damping, base);
+    }
+    INL_CUDA(cudaGetLastError());
+  }
+}
+
 void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damping, int iters,
                   float *rank) {
+  if (p->bins.flags & (kTemplateFlags | INL_BINS_THREAD_ONLY)) {
+    INL_CHECK(!has_comm(ctx), "pagerank: the paper's templates / T1 run on one GPU (no communicator)");
+    if (p->n_global == 0) return;
+    if (iters == 0) {
+      k_fill<<<grid_for(p->n_global, ctx->num_sms), 256, 0, ctx->stream>>>(rank, p->n_global,
+                                                                           (float)(1.0 / (double)p->n_global));
+      INL_CUDA(cudaGetLastError());
+      return;
+    }
+    pagerank_template(ctx, p, out_degree, damping, iters, rank);
+    return;
+  }
   cudaStream_t st = ctx->stream;
   const int64_t n = p->n_global;
   if (n == 0) return;

@@ -16,6 +16,7 @@
 //   * dbuf-shared: the buffer lives in shared memory; "a single kernel invocation but
 //     possibly leading to uneven work distribution among thread-blocks" —
 //     k_tpl_dbuf_shared.
+// val == nullptr: implicit unit values (PageRank's pull through the templates, pagerank.cu).
 // Row sums: serial in one thread (thread mapping) or strided over the CTA plus a fixed
 // shared-memory tree (block mapping): deterministic.  Queue order from atomics may vary;
 // each row's sum does not.
@@ -30,7 +31,7 @@ namespace {
 __device__ __forceinline__ float row_serial(const int64_t *rp, const int32_t *col, const float *val,
                                             const float *x, int64_t r) {
   float acc = 0.0f;
-  for (int64_t k = rp[r]; k < rp[r + 1]; ++k) acc += val[k] * __ldg(x + col[k]);
+  for (int64_t k = rp[r]; k < rp[r + 1]; ++k) acc += (val ? val[k] : 1.0f) * __ldg(x + col[k]);
   return acc;
 }
 
@@ -38,7 +39,8 @@ __device__ __forceinline__ float row_serial(const int64_t *rp, const int32_t *co
 __device__ __forceinline__ float row_block(const int64_t *rp, const int32_t *col, const float *val,
                                            const float *x, int64_t r, float *red) {
   float acc = 0.0f;
-  for (int64_t k = rp[r] + threadIdx.x; k < rp[r + 1]; k += blockDim.x) acc += val[k] * __ldg(x + col[k]);
+  for (int64_t k = rp[r] + threadIdx.x; k < rp[r + 1]; k += blockDim.x)
+    acc += (val ? val[k] : 1.0f) * __ldg(x + col[k]);
   for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
   const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   __syncthreads();  // red[] reuse

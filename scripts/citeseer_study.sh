@@ -13,4 +13,9 @@ for v in thread_only dual_queue:32:64 dbuf_global:32:64 dbuf_shared:32:64 dbuf_s
   f=$(echo $v | tr ': ()' '____')
   timeout 600 ncu --metrics $M --clock-control none --csv --log-file "gpurun_out/eff_spmv_$f.csv" python scripts/template_study.py --graph citeseer --only "$v" --reps 1 > /dev/null 2>&1
 done
+for v in thread_only dual_queue:32 dbuf_shared:32 dbuf_shared:64 dbuf_shared:256 dbuf_shared:1024 default; do
+  f=$(echo $v | tr ":" "_")
+  timeout 600 ncu --metrics $M --clock-control none --csv --log-file gpurun_out/eff_pr_$f.csv python scripts/template_study_pr.py --graph citeseer --only $v --iterations 3 > /dev/null 2>&1
+done
+timeout 900 python scripts/template_study_pr.py --graph citeseer > gpurun_out/ts_pr_citeseer.jsonl 2> gpurun_out/ts_pr_citeseer.err
 echo citeseer study done

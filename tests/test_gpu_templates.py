@@ -69,12 +69,24 @@ def test_template_uniform_and_star(ctx, g14, name):
     assert np.array_equal(run(ctx, rp, ci, n, v, xx, TPL[name], 16, 64), oracle.spmv(rp, ci, v, xx))
 
 
-def test_template_flags_are_spmv_only(ctx, g14):
+@pytest.mark.parametrize("name", ["thread_only", "dual_queue", "dbuf_global", "dbuf_shared"])
+@pytest.mark.parametrize("lbt", [8, 64])
+def test_pagerank_templates(ctx, name, lbt):
+    """PageRank through the paper's templates / its T1 baseline (template study, one GPU) vs the
+    20-iteration oracle, <= 1e-5."""
+    g = inlgen.host_build(14, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.TRANSPOSE)
+    A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
+    fl = inl.BINS_THREAD_ONLY if name == "thread_only" else TPL[name]
+    plan = inl.Plan(ctx, A, inl.bins(t_thread=lbt, t_warp=max(lbt, 16), t_block=max(lbt, 16), cta_threads=64,
+                                     flags=fl))
+    r = torch.empty(g.n_global, device="cuda")
+    inl.pagerank(ctx, A, dev(g.out_degree), r, 0.85, 20, plan)
+    ref = oracle.pagerank(g.n_global, g.row_ptr, g.col_idx, g.out_degree, 0.85, 20)
+    assert np.max(np.abs(r.cpu().numpy().astype(np.float64) - ref) / ref) <= 1e-5
+
+
+def test_template_flag_combinations(ctx, g14):
     A = inl.Csr(dev(g14.row_ptr), dev(g14.col_idx), g14.n_global)
-    plan = inl.Plan(ctx, A, inl.bins(flags=inl.BINS_TPL_DBUF_SHARED))
-    r = torch.empty(g14.n_global, device="cuda")
-    with pytest.raises(RuntimeError):
-        inl.pagerank(ctx, A, dev(np.ones(g14.n_global, np.int32)), r, 0.85, 2, plan)
     # more than one template, or a template with another flag: rejected when the plan is made
     for fl in (inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DUAL_QUEUE, inl.BINS_TPL_DUAL_QUEUE | inl.BINS_TPL_DBUF_GLOBAL,
                inl.BINS_TPL_DBUF_SHARED | inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DBUF_GLOBAL | inl.BINS_THREAD_ONLY):
