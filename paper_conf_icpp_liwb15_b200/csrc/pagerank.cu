@@ -329,10 +329,11 @@ static void pagerank_template(inl_ctx ctx, inl_plan p, const int32_t *od, float 
   cudaStream_t st = ctx->stream;
   const int64_t n = p->n_global;
   inl_csr A{p->n_rows, p->n_global, p->row_begin, p->nnz, p->row_ptr, p->col_idx};
-  float *c = (float *)ctx->s_a.get(sizeof(float) * (size_t)n);
-  float *s = (float *)ctx->s_b.get(sizeof(float) * (size_t)n);
+  // not s_a / s_b / s_f: spmv_template's queues and counters live there
+  float *c = (float *)ctx->s_d.get(sizeof(float) * (size_t)n);
+  float *s = (float *)ctx->s_e.get(sizeof(float) * (size_t)n);
   const int grid = grid_for(n, ctx->num_sms);
-  char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (size_t)grid);
+  char *scal = (char *)ctx->s_g.get(256 + sizeof(double) * (size_t)grid);
   float *base = (float *)scal;
   unsigned long long *ndang = (unsigned long long *)(scal + 8);
   double *dall = (double *)(scal + 16);
