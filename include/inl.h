@@ -249,7 +249,14 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
  *   bc[v] = sum_{s in sources} sum_{t != s, v} sigma_st(v) / sigma_st      (fp64)
  * bc [n_global] double (device or host), overwritten.  All vertices as sources = exact
  * BC (ordered pairs; an undirected graph's usual value is half).  One GPU (no row
- * blocks).  stats: iterations = forward levels over all sources.  Blocks until done. */
+ * blocks).  Two paths, chosen by a cost model (environment INL_BC_MODE=level|src forces one):
+ * level-synchronous (every source through grid-wide level steps, degree-binned, pull steps on
+ * a symmetric plan) and source-parallel (one CTA per source, both sweeps inside the CTA, state
+ * in shared memory when 20 B x n_global fits; for many sources on small graphs).  A plan whose
+ * bins.flags name one of the paper's templates (INL_BINS_TPL_*, lbTHRES = t_thread, CTA =
+ * cta_threads) or INL_BINS_THREAD_ONLY runs both sweeps of every level through that template
+ * (the template study).  Deterministic for a given path and source list.
+ * stats: iterations = forward levels over all sources.  Blocks until done. */
 inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t n_sources, double *bc,
                   inl_stats *stats, inl_plan plan);
 

@@ -228,6 +228,17 @@ def citeseer_like(seed: int = SEED_GRAPH) -> HostGraph:
     return powerlaw_build(CITESEER_N, CITESEER_DMIN, CITESEER_DMAX, CITESEER_MEAN, seed)
 
 
+# PAPER.md P5@13172-13524: Wiki-vote, 7,115 nodes, 103,689 edges, outdegree 0..893, mean 14.6
+# (reading R7: an undirected stand-in with the same n, entry count and degree range;
+# the configuration model needs dmin >= 1)
+WIKIVOTE_N, WIKIVOTE_DMIN, WIKIVOTE_DMAX, WIKIVOTE_MEAN = 7115, 1, 893, 14.6
+
+
+def wikivote_like(seed: int = SEED_GRAPH) -> HostGraph:
+    """The Wiki-vote-shaped synthetic graph of the BC template study (Fig. 6; symmetric CSR)."""
+    return powerlaw_build(WIKIVOTE_N, WIKIVOTE_DMIN, WIKIVOTE_DMAX, WIKIVOTE_MEAN, seed)
+
+
 def dev_build(scale: int, edge_factor: int = 16, seed: int = SEED_GRAPH, flags: int = 0,
               row_begin: int = 0, row_end: int = -1, device=None):
     """Device build (bit-identical to host_build); returns a dict of torch CUDA tensors."""

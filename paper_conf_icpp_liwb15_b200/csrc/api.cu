@@ -770,7 +770,8 @@ inl_status inl_bc(inl_ctx ctx, const inl_csr *G, const int64_t *sources, int64_t
     inl_csr d = device_csr(ctx, G);
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
     StagedOut<double> o = stage_out(ctx->h_y, bc, G->n_global);
-    bc_run(ctx, d, sources, n_sources, o.dev, stats, plan && plan->symmetric);
+    const Bins b = plan ? plan->bins : resolve_bins(nullptr);
+    bc_run(ctx, d, b, sources, n_sources, o.dev, stats, plan && plan->symmetric);
     finish_out(ctx, o);
     ctx_sync(ctx);
   });

@@ -16,7 +16,9 @@
 //                        one 16-B record (one gather per backward edge).
 #include <cooperative_groups.h>
 
+#include <algorithm>
 #include <cstdlib>
+#include <cstring>
 #include <vector>
 
 #include "inl_internal.cuh"
@@ -240,6 +242,316 @@ __global__ void __launch_bounds__(kBcNT) k_bc_pull(BcArgs a, int64_t n) {
   }
 }
 
+// ---- the paper's templates (template study, Fig. 6 BC bars / Table II BC row) ----------
+// Outer loop: the vertices Q[lo, hi) of one level; inner loop: their adjacency.  lbTHRES =
+// bins.t_thread, CTA size = bins.cta; forward and backward use the same mapping.
+//   T1 (INL_BINS_THREAD_ONLY): k_bct_thread over the whole level (thread-mapped, the
+//     paper's baseline); dual-queue: k_bct_split -> k_bct_thread (small) + k_bct_block
+//     (large); dbuf-global: k_bct_dbuf_global (defers large vertices to a global buffer) +
+//     k_bct_block; dbuf-shared: k_bct_dbuf_shared (shared buffer, same CTA).
+// Backward sums: thread-serial in edge order, block-mapped over a fixed CTA tree.
+
+// one vertex, thread-mapped (serial inner loop)
+template <bool FWD>
+__device__ __forceinline__ void bct_serial(const BcArgs &a, int32_t u) {
+  const int64_t rs = a.rp[u], re = a.rp[u + 1];
+  const double su = a.sigma[u];
+  if (FWD) {
+    for (int64_t k = rs; k < re; ++k) fwd_edge(a, su, __ldg(a.col + k));
+  } else {
+    double d = 0.0;
+    for (int64_t k = rs; k < re; ++k) d += bwd_term(a, su, __ldg(a.col + k));
+    bwd_finish(a, u, d);
+  }
+}
+
+// one vertex, block-mapped (threads stride the inner loop; backward: fixed CTA tree)
+template <bool FWD>
+__device__ __forceinline__ void bct_block(const BcArgs &a, int32_t u, double *red) {
+  const int64_t rs = a.rp[u], re = a.rp[u + 1];
+  const double su = a.sigma[u];
+  if (FWD) {
+    for (int64_t k = rs + threadIdx.x; k < re; k += blockDim.x) fwd_edge(a, su, __ldg(a.col + k));
+    return;
+  }
+  double d = 0.0;
+  for (int64_t k = rs + threadIdx.x; k < re; k += blockDim.x) d += bwd_term(a, su, __ldg(a.col + k));
+  for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+  __syncthreads();  // red[] reuse
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = d;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int q = 0; q < (int)(blockDim.x >> 5); ++q) t += red[q];
+    bwd_finish(a, u, t);
+  }
+}
+
+// dual-queue pre-pass over the level: degree <= lbt -> small queue, else large queue
+__global__ void k_bct_split(BcArgs a, int lbt, int32_t *qs, int *ns, int32_t *ql, int *nl) {
+  for (int i = a.lo + blockIdx.x * blockDim.x + threadIdx.x; i < a.hi; i += gridDim.x * blockDim.x) {
+    const int32_t u = a.Q[i];
+    if (a.rp[u + 1] - a.rp[u] <= lbt) qs[atomicAdd(ns, 1)] = u;
+    else ql[atomicAdd(nl, 1)] = u;
+  }
+}
+
+// thread mapping over a queue (q == nullptr: the level itself)
+template <bool FWD>
+__global__ void k_bct_thread(BcArgs a, const int32_t *q, const int *nq) {
+  const int n = q ? *nq : a.hi - a.lo;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    bct_serial<FWD>(a, q ? q[i] : a.Q[a.lo + i]);
+}
+
+// block mapping over a queue: one CTA per vertex, grid-stride (count read on the device)
+template <bool FWD>
+__global__ void k_bct_block(BcArgs a, const int32_t *q, const int *nq) {
+  __shared__ double red[32];
+  const int n = *(volatile const int *)nq;
+  for (int i = blockIdx.x; i < n; i += gridDim.x) bct_block<FWD>(a, q[i], red);
+}
+
+// dbuf-global phase 1: thread per level vertex; large ones go to a global buffer
+template <bool FWD>
+__global__ void k_bct_dbuf_global(BcArgs a, int lbt, int32_t *buf, int *nbuf) {
+  for (int i = a.lo + blockIdx.x * blockDim.x + threadIdx.x; i < a.hi; i += gridDim.x * blockDim.x) {
+    const int32_t u = a.Q[i];
+    if (a.rp[u + 1] - a.rp[u] <= lbt) bct_serial<FWD>(a, u);
+    else buf[atomicAdd(nbuf, 1)] = u;
+  }
+}
+
+// dbuf-shared: thread per level vertex; large ones queued in shared memory and run
+// block-mapped by the same CTA after __syncthreads
+template <bool FWD>
+__global__ void k_bct_dbuf_shared(BcArgs a, int lbt) {
+  extern __shared__ int32_t sbuf[];  // [blockDim.x]
+  __shared__ int ns;
+  __shared__ double red[32];
+  for (int i0 = a.lo + blockIdx.x * blockDim.x; i0 < a.hi; i0 += gridDim.x * blockDim.x) {
+    if (threadIdx.x == 0) ns = 0;
+    __syncthreads();
+    const int i = i0 + threadIdx.x;
+    if (i < a.hi) {
+      const int32_t u = a.Q[i];
+      if (a.rp[u + 1] - a.rp[u] <= lbt) bct_serial<FWD>(a, u);
+      else sbuf[atomicAdd(&ns, 1)] = u;
+    }
+    __syncthreads();
+    const int m = ns;
+    for (int j = 0; j < m; ++j) bct_block<FWD>(a, sbuf[j], red);
+    __syncthreads();
+  }
+}
+
+// ---- source-parallel BC (many sources): one CTA per source -------------------------------
+// The paper's BC runs every source through grid-wide level steps (a launch pair and a host
+// sync per level).  With many sources and a graph whose per-source state fits one SM, the
+// sources themselves are the outer parallel loop: CTA c runs sources c, c + G, c + 2G, ...
+// (static, so the result is deterministic), each with both sweeps inside the CTA
+// (__syncthreads between levels, no launches, no host syncs).  The level's nested loop keeps
+// the paper's binning inside the CTA (dbuf-shared, P5@3623): a thread per frontier vertex,
+// degree > kSrcThread deferred to shared lists run by 8-lane groups (<= kSrcGroup) or warps.
+// State per CTA — level int32, sigma f64, coef f64 ((1 + delta) / sigma of a finished
+// vertex) — sits in shared memory when 20 B x n fits (SMEM), else in global slices
+// (L2-resident for small n); the visit order Q and the level offsets are global; bc partial
+// sums per CTA (bc_part[c][v], plain stores) are added in CTA order by k_bc_src_reduce.
+constexpr int kSrcNT = 1024;
+constexpr int kSrcThread = 4;
+constexpr int kSrcGroup = 64;
+
+struct SrcArgs {
+  const int64_t *rp;
+  const int32_t *col;
+  int32_t n;
+  const int32_t *sources;
+  int32_t n_sources;
+  int32_t *g_level;          // [G][n] (global state only)
+  double *g_sigma, *g_coef;  // [G][n]
+  int32_t *g_Q;              // [G][n]
+  int32_t *g_off;            // [G][n + 2] level offsets into Q
+  double *bc_part;           // [G][n]
+  unsigned long long *levels;   // forward levels over all sources (stats)
+  unsigned long long *reached;  // vertices reached over all sources (stats)
+};
+
+__device__ __forceinline__ void src_enqueue(int32_t *Q, int *tail, int32_t v) {
+  cg::coalesced_group g = cg::coalesced_threads();
+  int pos = 0;
+  if (g.thread_rank() == 0) pos = atomicAdd(tail, (int)g.size());
+  pos = g.shfl(pos, 0) + (int)g.thread_rank();
+  Q[pos] = v;
+}
+
+// per-CTA state of one source's sweeps
+struct SrcState {
+  int32_t *level;
+  double *sigma, *coef;
+  int32_t *Q;
+  int *tail;
+  int L;
+};
+
+// forward edge u (level L, sigma su) -> v
+__device__ __forceinline__ void src_fwd(const SrcState &S, double su, int32_t v) {
+  int lv = ((volatile int32_t *)S.level)[v];
+  if (lv == -1) {
+    if (atomicCAS(S.level + v, -1, S.L + 1) == -1) src_enqueue(S.Q, S.tail, v);
+    lv = S.L + 1;
+  }
+  if (lv == S.L + 1) atomicAdd(S.sigma + v, su);
+}
+
+// backward term of edge w -> v (sw = sigma[w]); S.L = level of w
+__device__ __forceinline__ double src_bwd(const SrcState &S, double sw, int32_t v) {
+  return S.level[v] == S.L + 1 ? sw * S.coef[v] : 0.0;
+}
+
+__device__ __forceinline__ void src_finish(const SrcState &S, double *part, int32_t w, double sw, double d) {
+  S.coef[w] = (1.0 + d) / sw;
+  part[w] += d;
+}
+
+// one level (forward: FWD) of the CTA's source over Q[lo, hi): thread / 8-lane group / warp
+template <bool FWD>
+__device__ __forceinline__ void src_level(const SrcArgs &a, const SrcState &S, double *part, int lo, int hi,
+                                          int32_t *gl, int32_t *wl, int *ng, int *nw, int &ph) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (int base = lo; base < hi; base += kSrcNT) {
+    const int i = base + tid;
+    if (i < hi) {
+      const int32_t u = S.Q[i];
+      const int64_t rs = a.rp[u], re = a.rp[u + 1];
+      if (re - rs <= kSrcThread) {
+        const double su = S.sigma[u];
+        if (FWD) {
+          for (int64_t k = rs; k < re; ++k) src_fwd(S, su, __ldg(a.col + k));
+        } else {
+          double d = 0.0;
+          for (int64_t k = rs; k < re; ++k) d += src_bwd(S, su, __ldg(a.col + k));
+          src_finish(S, part, u, su, d);
+        }
+      } else if (re - rs <= kSrcGroup) {
+        gl[atomicAdd(&ng[ph], 1)] = u;
+      } else {
+        wl[atomicAdd(&nw[ph], 1)] = u;
+      }
+    }
+    __syncthreads();
+    const int mg = ng[ph], mw = nw[ph];
+    if (tid == 0) ng[ph ^ 1] = nw[ph ^ 1] = 0;  // the other pair is reset for the next chunk
+    const int sub = lane & 7, grp = lane >> 3;
+    for (int j0 = warp * 4; j0 < mg; j0 += kSrcNT / 8) {  // 8-lane groups (warp-uniform rounds)
+      const int j = j0 + grp;
+      double d = 0.0, su = 0.0;
+      int32_t u = -1;
+      if (j < mg) {
+        u = gl[j];
+        su = S.sigma[u];
+        for (int64_t k = a.rp[u] + sub; k < a.rp[u + 1]; k += 8) {
+          if (FWD) src_fwd(S, su, __ldg(a.col + k));
+          else d += src_bwd(S, su, __ldg(a.col + k));
+        }
+      }
+      if (!FWD) {
+        for (int o = 4; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+        if (sub == 0 && u >= 0) src_finish(S, part, u, su, d);
+      }
+    }
+    for (int j = warp; j < mw; j += kSrcNT / 32) {  // warps
+      const int32_t u = wl[j];
+      const double su = S.sigma[u];
+      double d = 0.0;
+      for (int64_t k = a.rp[u] + lane; k < a.rp[u + 1]; k += 32) {
+        if (FWD) src_fwd(S, su, __ldg(a.col + k));
+        else d += src_bwd(S, su, __ldg(a.col + k));
+      }
+      if (!FWD) {
+        for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+        if (lane == 0) src_finish(S, part, u, su, d);
+      }
+    }
+    __syncthreads();
+    ph ^= 1;
+  }
+}
+
+template <bool SMEM>
+__global__ void __launch_bounds__(kSrcNT, 1) k_bc_src(SrcArgs a) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  __shared__ int32_t gl[kSrcNT], wl[kSrcNT];
+  __shared__ int ng[2], nw[2], tail;  // list counters: ping-pong per chunk
+  const int tid = threadIdx.x;
+  const int n = a.n;
+  const size_t c = blockIdx.x;
+  SrcState S;
+  if (SMEM) {
+    S.sigma = (double *)sm;
+    S.coef = S.sigma + n;
+    S.level = (int32_t *)(S.coef + n);
+  } else {
+    S.level = a.g_level + c * n;
+    S.sigma = a.g_sigma + c * n;
+    S.coef = a.g_coef + c * n;
+  }
+  S.Q = a.g_Q + c * n;
+  S.tail = &tail;
+  int32_t *off = a.g_off + c * (size_t)(n + 2);
+  double *part = a.bc_part + c * n;
+  for (int v = tid; v < n; v += kSrcNT) part[v] = 0.0;
+  unsigned long long nlev = 0, nreach = 0;
+  int ph = 0;
+  for (int si = blockIdx.x; si < a.n_sources; si += gridDim.x) {
+    const int32_t s = a.sources[si];
+    for (int v = tid; v < n; v += kSrcNT) {
+      S.level[v] = v == s ? 0 : -1;
+      S.sigma[v] = v == s ? 1.0 : 0.0;
+    }
+    if (tid == 0) {
+      S.Q[0] = s;
+      off[0] = 0;
+      off[1] = 1;
+      tail = 1;
+      ng[0] = ng[1] = nw[0] = nw[1] = 0;
+    }
+    __syncthreads();
+    int L = 0, lo = 0, hi = 1;
+    while (lo < hi) {  // forward: level L = Q[lo, hi)
+      S.L = L;
+      src_level<true>(a, S, part, lo, hi, gl, wl, ng, nw, ph);
+      lo = hi;
+      hi = *(volatile int *)&tail;
+      ++L;
+      if (tid == 0) off[L + 1] = hi;
+      __syncthreads();  // everyone has read tail before the next level appends
+    }
+    if (tid == 0) {
+      nlev += L;
+      nreach += lo;
+    }
+    // levels 0 .. L-1 are non-empty; backward from the deepest, level 0 (the source) skipped
+    for (int l = L - 1; l >= 1; --l) {
+      S.L = l;
+      src_level<false>(a, S, part, off[l], off[l + 1], gl, wl, ng, nw, ph);
+    }
+    __syncthreads();
+  }
+  if (tid == 0 && nlev) {
+    atomicAdd(a.levels, nlev);
+    atomicAdd(a.reached, nreach);
+  }
+}
+
+// bc[v] = sum over CTAs c (in order) of bc_part[c][v]
+__global__ void k_bc_src_reduce(const double *__restrict__ part, int G, int64_t n, double *bc) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    double t = 0.0;
+    for (int c = 0; c < G; ++c) t += part[(size_t)c * n + v];
+    bc[v] = t;
+  }
+}
+
 __global__ void k_bc_init(int32_t *level, double *sigma, int64_t n, int64_t s, int32_t *Q) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
     level[v] = v == s ? 0 : -1;
@@ -259,14 +571,116 @@ int grid_of(int64_t n, int sms) {
   return g < 1 ? 1 : (int)g;
 }
 
+
+// shared-memory bytes of one CTA's state (sigma, coef, level), 0 if it does not fit
+size_t src_smem_bytes(inl_ctx ctx, int64_t n) {
+  static int optin[kMaxDevices] = {};
+  int &o = optin[ctx->device % kMaxDevices];
+  if (!o) INL_CUDA(cudaDeviceGetAttribute(&o, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device));
+  const size_t need = (size_t)n * 20;
+  const size_t stat = 2 * sizeof(int32_t) * kSrcNT + 1024 + 64;  // k_bc_src static + reserved shared memory
+  return need + stat <= (size_t)o ? need : 0;
+}
+
+// global scratch bytes per CTA of the source-parallel path
+size_t src_global_bytes(int64_t n, bool smem) {
+  return (size_t)n * (smem ? 16 : 36) + 8 * 2 + 16;
+}
+
+// Source-parallel when its modelled time beats the level-synchronous path's (INL_BC_MODE=
+// level|src overrides).  Model fitted to profiles/r02/bc_mode_sweep.jsonl (B200, symmetric
+// R-MAT 14..20 and the Wiki-vote-shaped graph): one source on one SM costs ~3.3 ns per CSR
+// entry while the per-CTA state stays in L2 (~6 ns beyond), the sources run ceil(ns / G)
+// deep; a level-synchronous source costs max(0.4 ms (launches + a host sync per level),
+// 0.033 ns per entry).
+bool bc_use_src(inl_ctx ctx, const inl_csr &G, int64_t n_sources) {
+  const char *e = getenv("INL_BC_MODE");
+  if (e && !strcmp(e, "level")) return false;
+  const int64_t n = G.n_global;
+  const int64_t Gc = std::min<int64_t>(n_sources, ctx->num_sms);
+  const bool smem = src_smem_bytes(ctx, n) > 0;
+  const double bytes = (double)Gc * (double)src_global_bytes(n, smem);
+  const bool fits = n < INT32_MAX && n_sources < INT32_MAX && bytes <= 4.0e9;
+  if (e && !strcmp(e, "src")) {
+    INL_CHECK(fits, "INL_BC_MODE=src: the per-CTA state does not fit");
+    return true;
+  }
+  if (!fits) return false;
+  const double nnz = (double)G.nnz;
+  const double per_edge = smem || bytes <= 64.0e6 ? 3.3e-9 : 6.0e-9;
+  const double t_src = (double)((n_sources + Gc - 1) / Gc) * nnz * per_edge;
+  const double t_level = (double)n_sources * std::max(0.4e-3, nnz * 0.033e-9);
+  return t_src < t_level;
+}
+
+void bc_src_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
+                inl_stats *stats) {
+  cudaStream_t st = ctx->stream;
+  const int64_t n = G.n_global;
+  const int Gc = (int)std::min<int64_t>(n_sources, ctx->num_sms);
+  const size_t smem = src_smem_bytes(ctx, n);
+  SrcArgs a{};
+  a.rp = G.row_ptr;
+  a.col = G.col_idx;
+  a.n = (int32_t)n;
+  a.n_sources = (int32_t)n_sources;
+  std::vector<int32_t> hs((size_t)n_sources);
+  for (int64_t i = 0; i < n_sources; ++i) hs[(size_t)i] = (int32_t)sources[i];
+  int32_t *dsrc = (int32_t *)ctx->s_tmp.get(sizeof(int32_t) * n_sources);
+  INL_CUDA(cudaMemcpyAsync(dsrc, hs.data(), sizeof(int32_t) * n_sources, cudaMemcpyHostToDevice, st));
+  a.sources = dsrc;
+  const size_t gn = (size_t)Gc * n;
+  a.bc_part = (double *)ctx->s_a.get(sizeof(double) * gn);
+  a.g_Q = (int32_t *)ctx->s_b.get(sizeof(int32_t) * gn);
+  a.g_off = (int32_t *)ctx->s_c.get(sizeof(int32_t) * (size_t)Gc * (n + 2));
+  if (!smem) {
+    a.g_sigma = (double *)ctx->s_d.get(sizeof(double) * gn);
+    a.g_coef = (double *)ctx->s_e.get(sizeof(double) * gn);
+    a.g_level = (int32_t *)ctx->s_g.get(sizeof(int32_t) * gn);
+  }
+  unsigned long long *cnt = (unsigned long long *)ctx->s_f.get(64);
+  a.levels = cnt;
+  a.reached = cnt + 1;
+  INL_CUDA(cudaMemsetAsync(cnt, 0, 16, st));
+  static size_t configured[kMaxDevices] = {};
+  size_t &cf = configured[ctx->device % kMaxDevices];
+  if (smem > cf) {
+    INL_CUDA(cudaFuncSetAttribute(k_bc_src<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cf = smem;
+  }
+  {
+    KScope ks(ctx, "k_bc_src");
+    if (smem) k_bc_src<true><<<Gc, kSrcNT, smem, st>>>(a);
+    else k_bc_src<false><<<Gc, kSrcNT, 0, st>>>(a);
+    INL_CUDA(cudaGetLastError());
+  }
+  k_bc_src_reduce<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(a.bc_part, Gc, n, bc);
+  INL_CUDA(cudaGetLastError());
+  INL_CUDA(cudaMemcpyAsync(ctx->pinned, cnt, 16, cudaMemcpyDeviceToHost, st));
+  INL_CUDA(cudaStreamSynchronize(st));
+  if (stats) {
+    stats->iterations = (int32_t)((volatile unsigned long long *)ctx->pinned)[0];
+    stats->edges_relaxed = 0;
+    stats->frontier_total = (int64_t)((volatile unsigned long long *)ctx->pinned)[1];
+    stats->launches = 2;
+    stats->host_syncs = 0;
+    stats->exchange_bytes = 0;
+  }
+}
+
 }  // namespace
 
-void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
+void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources, int64_t n_sources, double *bc,
             inl_stats *stats, bool symmetric) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   INL_CHECK(n < INT32_MAX, "bc: n must be < 2^31");
   if (n == 0) return;
+  const int tpl = b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags);
+  if (!tpl && n_sources > 0 && bc_use_src(ctx, G, n_sources)) {
+    bc_src_run(ctx, G, sources, n_sources, bc, stats);
+    return;
+  }
   int32_t *level = (int32_t *)ctx->s_a.get(sizeof(int32_t) * n);
   int32_t *Q = (int32_t *)ctx->s_b.get(sizeof(int32_t) * (n + 1));
   double *sigma = (double *)ctx->s_c.get(sizeof(double) * n);
@@ -294,6 +708,49 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
     pull_edge = 0.5;  // measured on one box at scale 22: n/8 rule 5.38, 0.5 -> 4.16, 1 -> 4.34, 2 -> 5.64 ms
     if (const char *e = getenv("INL_BC_PULL_EDGE")) pull_edge = atof(e);
   }
+  // the paper's templates / T1 baseline (bins flags): plain push levels, no pull
+  if (tpl) symmetric = false;
+  int32_t *tq = tpl == INL_BINS_TPL_DUAL_QUEUE || tpl == INL_BINS_TPL_DBUF_GLOBAL
+                    ? (int32_t *)ctx->s_h.get(sizeof(int32_t) * 2 * n) : nullptr;
+  // one level of either sweep through the template; returns the launches
+  auto tpl_level = [&](const BcArgs &a, bool fwd) -> int {
+    const int m = a.hi - a.lo, cta = b.cta, lbt = b.t_thread, sms = ctx->num_sms;
+    int g = (m + cta - 1) / cta;
+    if (g > sms * 32) g = sms * 32;
+    int *tc = cnt + 8;  // template queue counters
+    if (tpl == INL_BINS_THREAD_ONLY) {
+      if (fwd) k_bct_thread<true><<<g, cta, 0, st>>>(a, nullptr, nullptr);
+      else k_bct_thread<false><<<g, cta, 0, st>>>(a, nullptr, nullptr);
+      return 1;
+    }
+    if (tpl == INL_BINS_TPL_DBUF_SHARED) {
+      if (fwd) k_bct_dbuf_shared<true><<<g, cta, sizeof(int32_t) * cta, st>>>(a, lbt);
+      else k_bct_dbuf_shared<false><<<g, cta, sizeof(int32_t) * cta, st>>>(a, lbt);
+      return 1;
+    }
+    INL_CUDA(cudaMemsetAsync(tc, 0, 2 * sizeof(int), st));
+    if (tpl == INL_BINS_TPL_DUAL_QUEUE) {
+      int gs = (m + 255) / 256;
+      if (gs > sms * 16) gs = sms * 16;
+      k_bct_split<<<gs, 256, 0, st>>>(a, lbt, tq, tc, tq + n, tc + 1);
+      if (fwd) {
+        k_bct_thread<true><<<g, cta, 0, st>>>(a, tq, tc);
+        k_bct_block<true><<<sms * 16, cta, 0, st>>>(a, tq + n, tc + 1);
+      } else {
+        k_bct_thread<false><<<g, cta, 0, st>>>(a, tq, tc);
+        k_bct_block<false><<<sms * 16, cta, 0, st>>>(a, tq + n, tc + 1);
+      }
+      return 3;
+    }
+    if (fwd) {
+      k_bct_dbuf_global<true><<<g, cta, 0, st>>>(a, lbt, tq, tc);
+      k_bct_block<true><<<sms * 16, cta, 0, st>>>(a, tq, tc);
+    } else {
+      k_bct_dbuf_global<false><<<g, cta, 0, st>>>(a, lbt, tq, tc);
+      k_bct_block<false><<<sms * 16, cta, 0, st>>>(a, tq, tc);
+    }
+    return 2;
+  };
   for (int64_t si = 0; si < n_sources; ++si) {
     const int64_t s = sources[si];
     k_bc_init<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(level, sigma, n, s, Q);
@@ -311,7 +768,10 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
       INL_CUDA(cudaMemsetAsync(cnt, 0, 24, st));  // counters + m_f
       const bool pull = symmetric && (pull_edge > 0.0 ? (double)mf_next * pull_edge > m_u
                                                       : pull_div > 0 && (int64_t)(a.hi - a.lo) * pull_div > n);
-      if (pull) {  // large frontier: pull from the unvisited side
+      if (tpl) {
+        KScope ks(ctx, "k_bc_fwd");
+        launches += tpl_level(a, true);
+      } else if (pull) {  // large frontier: pull from the unvisited side
         KScope ks(ctx, "k_bc_fwd");
         k_bc_pull<<<ctx->num_sms * 8, kBcNT, 0, st>>>(a, n);
         launches += 1;
@@ -321,7 +781,7 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
         k_bc_big<true><<<ctx->num_sms * 4, kBcNT, 0, st>>>(a);
         launches += 2;
       }
-      if (pull_edge > 0.0) {
+      if (pull_edge > 0.0 && !tpl) {
         k_bc_degsum<<<ctx->num_sms * 2, 256, 0, st>>>(a);
         ++launches;
       }
@@ -341,6 +801,12 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sou
       a.lo = off[L];
       a.hi = off[L + 1];
       a.L = L;
+      if (tpl) {
+        KScope ks(ctx, "k_bc_bwd");
+        launches += tpl_level(a, false);
+        INL_CUDA(cudaGetLastError());
+        continue;
+      }
       INL_CUDA(cudaMemsetAsync(cnt + 1, 0, 2 * sizeof(int), st));
       {
         KScope ks(ctx, "k_bc_bwd");

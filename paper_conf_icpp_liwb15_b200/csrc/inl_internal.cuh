@@ -253,7 +253,7 @@ void cb_build(inl_plan p, CbPlan &cb, const int32_t *cols, int64_t ncols, bool s
 void tree_run(inl_ctx ctx, const inl_csr &T, const int32_t *parent, int64_t root, int method, bool heights,
               int64_t *out, inl_stats *stats);
 // bc.cu
-void bc_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n_sources, double *bc,
+void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources, int64_t n_sources, double *bc,
             inl_stats *stats, bool symmetric);
 // validate
 void csr_validate(inl_ctx ctx, const inl_csr &A);

@@ -45,8 +45,18 @@ def main():
         inl.bfs(ctx, As, src, d, pt)
     bc = torch.empty(s.n_global, dtype=torch.float64, device="cuda")
     srcs = inlgen.sources(s.row_ptr, 3)
+    os.environ["INL_BC_MODE"] = "level"
     inl.bc(ctx, As, srcs, bc)
-    inl.bc(ctx, As, srcs, bc, ps)
+    inl.bc(ctx, As, srcs, bc, ps)  # pull steps
+    os.environ["INL_BC_MODE"] = "src"
+    inl.bc(ctx, As, srcs, bc)  # source-parallel, state in shared memory
+    s14 = inlgen.host_build(14, 8, seed=1, flags=inlgen.SYMMETRIC)
+    A14 = inl.Csr(dev(s14.row_ptr), dev(s14.col_idx), s14.n_global)
+    b14 = torch.empty(s14.n_global, dtype=torch.float64, device="cuda")
+    inl.bc(ctx, A14, inlgen.sources(s14.row_ptr, 3), b14)  # source-parallel, global state
+    del os.environ["INL_BC_MODE"]
+    for fl in (inl.BINS_TPL_DBUF_SHARED, inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DUAL_QUEUE, inl.BINS_THREAD_ONLY):
+        inl.bc(ctx, As, srcs, bc, inl.Plan(ctx, As, inl.bins(t_thread=16, cta_threads=128, flags=fl)))
     # the paper's templates and the column-blocked bin (small blocks: several per row)
     val, x = dev(inlgen.values_host(g.row_ptr, g.col_idx)), dev(inlgen.vector_host(g.n_global))
     for fl in (inl.BINS_TPL_DUAL_QUEUE, inl.BINS_TPL_DBUF_GLOBAL, inl.BINS_TPL_DBUF_SHARED):

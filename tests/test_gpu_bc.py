@@ -26,6 +26,13 @@ def ctx():
     return inl.Ctx(0)
 
 
+@pytest.fixture(params=["level", "src"])
+def mode(request, monkeypatch):
+    """Both non-template paths: level-synchronous, source-parallel (bc.cu)."""
+    monkeypatch.setenv("INL_BC_MODE", request.param)
+    return request.param
+
+
 def gpu_bc(ctx, rp, ci, n, sources):
     out = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
     st = inl.bc(ctx, inl.Csr(dev(rp), dev(ci), n), sources, out)
@@ -39,7 +46,7 @@ def check(got, ref):
         assert np.max(np.abs(got[~z] - ref[~z]) / ref[~z]) <= RTOL
 
 
-def test_closed_forms(ctx):
+def test_closed_forms(ctx, mode):
     n = 40
     rp, ci, _ = csr_from_edges(n, [(i, i + 1) for i in range(n - 1)], symmetric=True)
     got, _ = gpu_bc(ctx, rp, ci, n, range(n))
@@ -55,14 +62,14 @@ def test_closed_forms(ctx):
     assert np.all(gpu_bc(ctx, rp, ci, n, range(n))[0] == 0)
 
 
-def test_cfg1_exact_all_sources(ctx):
+def test_cfg1_exact_all_sources(ctx, mode):
     g = inlgen.host_build(12, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
     got, st = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, range(g.n_global))
     check(got, oracle.bc(g.row_ptr, g.col_idx))
     assert st["iterations"] >= g.n_global
 
 
-def test_directed_and_repeatable(ctx):
+def test_directed_and_repeatable(ctx, mode):
     g = inlgen.host_build(13, 16, seed=inlgen.SEED_GRAPH)  # directed R-MAT
     srcs = inlgen.sources(g.row_ptr, 16)
     got, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
@@ -71,14 +78,14 @@ def test_directed_and_repeatable(ctx):
     assert np.array_equal(got, again)
 
 
-def test_scale16_sources(ctx):
+def test_scale16_sources(ctx, mode):
     g = inlgen.host_build(16, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
     srcs = inlgen.sources(g.row_ptr, 8)
     got, _ = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
     check(got, oracle.bc(g.row_ptr, g.col_idx, srcs))
 
 
-def test_random_small_and_edge_cases(ctx):
+def test_random_small_and_edge_cases(ctx, mode):
     rng = np.random.default_rng(3)
     for trial in range(30):
         n = int(rng.integers(1, 40))
@@ -97,8 +104,9 @@ def test_random_small_and_edge_cases(ctx):
         gpu_bc(ctx, rp, ci, 4, [4])
 
 
-def test_pull_steps_with_symmetric_plan(ctx):
+def test_pull_steps_with_symmetric_plan(ctx, monkeypatch):
     """With a plan that verified symmetry, large frontiers are expanded by pull steps."""
+    monkeypatch.setenv("INL_BC_MODE", "level")
     g = inlgen.host_build(15, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
     A = inl.Csr(dev(g.row_ptr), dev(g.col_idx), g.n_global)
     plan = inl.Plan(ctx, A)
@@ -117,3 +125,108 @@ def test_pull_steps_with_symmetric_plan(ctx):
     s = inlgen.sources(d.row_ptr, 4)
     inl.bc(ctx, Ad, s, out, pd)
     check(out.cpu().numpy(), oracle.bc(d.row_ptr, d.col_idx, s))
+
+
+TEMPLATES = {"thread_only": inl.BINS_THREAD_ONLY, "dual_queue": inl.BINS_TPL_DUAL_QUEUE,
+             "dbuf_global": inl.BINS_TPL_DBUF_GLOBAL, "dbuf_shared": inl.BINS_TPL_DBUF_SHARED}
+
+
+def tpl_bc(ctx, h, srcs, flags, lbt, cta=192):
+    A = inl.Csr(dev(h.row_ptr), dev(h.col_idx), h.n_global)
+    plan = inl.Plan(ctx, A, inl.bins(t_thread=lbt, cta_threads=cta, flags=flags))
+    out = torch.full((h.n_global,), float("nan"), dtype=torch.float64, device="cuda")
+    st = inl.bc(ctx, A, srcs, out, plan)
+    return out.cpu().numpy(), st
+
+
+@pytest.mark.parametrize("name", sorted(TEMPLATES))
+@pytest.mark.parametrize("lbt", [1, 32, 1024])
+def test_templates_wikivote_shaped(ctx, name, lbt):
+    """Fig. 6 BC bars: the paper's templates (and T1) over lbTHRES on the Wiki-vote-shaped
+    graph; thread-serial vertices and CTA-tree vertices both appear at lbt 1 and 32."""
+    h = inlgen.wikivote_like()
+    srcs = inlgen.sources(h.row_ptr, 6)
+    got, st = tpl_bc(ctx, h, srcs, TEMPLATES[name], lbt)
+    check(got, oracle.bc(h.row_ptr, h.col_idx, srcs))
+    assert st["iterations"] >= len(srcs)
+
+
+@pytest.mark.parametrize("name", sorted(TEMPLATES))
+def test_templates_star_path_and_directed(ctx, name):
+    k = 3000  # the hub is block-mapped under every template but T1
+    rp, ci, _ = csr_from_edges(k + 1, [(0, i) for i in range(1, k + 1)], symmetric=True)
+    h = inlgen.HostGraph(k + 1, 0, rp, ci)
+    srcs = list(range(0, k + 1, 97))
+    got, _ = tpl_bc(ctx, h, srcs, TEMPLATES[name], 16, 128)
+    ref = oracle.bc(rp, ci, srcs)
+    check(got, ref)
+    n = 50
+    rp, ci, _ = csr_from_edges(n, [(i, i + 1) for i in range(n - 1)], symmetric=True)
+    got, _ = tpl_bc(ctx, inlgen.HostGraph(n, 0, rp, ci), range(n), TEMPLATES[name], 1, 64)
+    assert np.array_equal(got, [2.0 * i * (n - 1 - i) for i in range(n)])
+    d = inlgen.host_build(13, 16, seed=inlgen.SEED_GRAPH)  # directed R-MAT
+    s = inlgen.sources(d.row_ptr, 4)
+    got, _ = tpl_bc(ctx, d, s, TEMPLATES[name], 32, 256)
+    check(got, oracle.bc(d.row_ptr, d.col_idx, s))
+
+
+# ---- source-parallel BC (one CTA per source; bc.cu k_bc_src) -------------------------------
+
+@pytest.fixture
+def src_mode(monkeypatch):
+    monkeypatch.setenv("INL_BC_MODE", "src")
+
+
+def test_source_parallel_wikivote_auto(ctx):
+    """Many sources on the Wiki-vote-shaped graph: the auto choice is the source-parallel
+    kernel (state in shared memory), one launch pair, no host sync per level."""
+    h = inlgen.wikivote_like()
+    srcs = inlgen.sources(h.row_ptr, 300)
+    got, st = gpu_bc(ctx, h.row_ptr, h.col_idx, h.n_global, srcs)
+    assert st["launches"] == 2 and st["host_syncs"] == 0
+    check(got, oracle.bc(h.row_ptr, h.col_idx, srcs))
+    again, _ = gpu_bc(ctx, h.row_ptr, h.col_idx, h.n_global, srcs)
+    assert np.array_equal(got, again)  # static source -> CTA assignment, CTA-ordered reduction
+    g = inlgen.host_build(18, 16, seed=inlgen.SEED_GRAPH, flags=inlgen.SYMMETRIC)
+    s8 = inlgen.sources(g.row_ptr, 8)  # few sources on a larger graph: level-synchronous
+    got, st2 = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, s8)
+    assert st2["launches"] > 2
+    check(got, oracle.bc(g.row_ptr, g.col_idx, s8))
+
+
+def test_source_parallel_closed_forms(ctx, src_mode):
+    n = 40
+    rp, ci, _ = csr_from_edges(n, [(i, i + 1) for i in range(n - 1)], symmetric=True)
+    got, st = gpu_bc(ctx, rp, ci, n, range(n))
+    assert np.array_equal(got, [2.0 * i * (n - 1 - i) for i in range(n)])
+    assert st["iterations"] == sum(max(i, n - 1 - i) + 1 for i in range(n))
+    k = 5000  # hub: warp-mapped inside the CTA in both sweeps
+    rp, ci, _ = csr_from_edges(k + 1, [(0, i) for i in range(1, k + 1)], symmetric=True)
+    got, _ = gpu_bc(ctx, rp, ci, k + 1, range(0, k + 1, 7))
+    ref = oracle.bc(rp, ci, range(0, k + 1, 7))
+    check(got, ref)
+    assert got[0] == ref[0]
+
+
+@pytest.mark.parametrize("scale", [13, 14])  # 13: state in shared memory; 14: global slices
+def test_source_parallel_rmat(ctx, src_mode, scale):
+    for flags in (0, inlgen.SYMMETRIC):
+        g = inlgen.host_build(scale, 16, seed=inlgen.SEED_GRAPH, flags=flags)
+        srcs = inlgen.sources(g.row_ptr, 200)
+        got, st = gpu_bc(ctx, g.row_ptr, g.col_idx, g.n_global, srcs)
+        check(got, oracle.bc(g.row_ptr, g.col_idx, srcs))
+        assert st["launches"] == 2
+
+
+def test_source_parallel_edge_cases(ctx, src_mode):
+    rng = np.random.default_rng(5)
+    for trial in range(20):
+        n = int(rng.integers(1, 40))
+        e = [(int(rng.integers(n)), int(rng.integers(n))) for _ in range(int(rng.integers(0, 4 * n)))]
+        rp, ci, _ = csr_from_edges(n, e, symmetric=bool(trial % 2))
+        srcs = [int(v) for v in rng.integers(0, n, size=7)]  # repeats allowed
+        got, _ = gpu_bc(ctx, rp, ci, n, srcs)
+        check(got, oracle.bc(rp, ci, srcs))
+    rp, ci, _ = csr_from_edges(5, [], symmetric=True)  # edgeless: every source isolated
+    got, st = gpu_bc(ctx, rp, ci, 5, range(5))
+    assert np.all(got == 0) and st["iterations"] == 5

@@ -145,3 +145,15 @@ def test_citeseer_like_shape():
     assert deg.max() <= 1188 and np.mean(deg >= 1) > 0.999
     assert abs(deg.mean() - 73.9) / 73.9 < 0.02
     assert abs(len(g.col_idx) - 32.1e6) / 32.1e6 < 0.02
+
+
+def test_wikivote_like_shape():
+    """PAPER.md P5@13172-13524: Wiki-vote, 7,115 nodes, 103,689 edges, mean outdegree 14.6,
+    at most 893 (symmetric stand-in, R7)."""
+    g = inlgen.wikivote_like()
+    deg = np.diff(g.row_ptr)
+    assert g.n_global == 7115
+    assert deg.min() >= 1 and deg.max() <= 893
+    assert abs(deg.mean() - 14.6) / 14.6 < 0.02
+    assert abs(len(g.col_idx) - 103689) / 103689 < 0.02
+    assert np.array_equal(inlgen.wikivote_like().col_idx, g.col_idx)  # seeded
