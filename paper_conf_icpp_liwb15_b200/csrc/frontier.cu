@@ -99,6 +99,17 @@ struct SsspOp {
   int64_t B = 0;
   unsigned int *nimp = nullptr;
   unsigned long long *xops = nullptr;  // remote atomics issued (the exchange volume)
+  // bitmap frontier (the one-GPU graph loop): an improvement is a fire-and-forget atomicMin
+  // plus a fire-and-forget bit in the next-frontier (nbits) or far (fbits) bitmap — no
+  // queue counter, no atomic whose result a warp waits for; k_sssp_bcompact turns the bits
+  // into the next step's worklist.  A lost race only adds a vertex to the frontier (it is
+  // expanded with its true distance then), never loses an improvement.
+  uint32_t *nbits = nullptr;
+  uint32_t *fbits = nullptr;
+  __device__ __forceinline__ void mark(int32_t v, uint32_t nd) const {
+    red_min_u32(dist + v, nd);
+    red_or_b32((nd >= thr ? fbits : nbits) + (v >> 5), 1u << (v & 31));
+  }
   __device__ __forceinline__ bool xrelax(int32_t v, uint32_t nd) const {
     uint32_t *o = xd[v / B];
     if (o != dist) atomicMin(dist + v, nd);  // keep the local filter tight
@@ -118,6 +129,10 @@ struct SsspOp {
       const bool imp = xrelax(v, nd);
       if (imp) atomicAdd(nimp, 1u);
       if (r) atomicAdd(xops, imp ? 2ull : 1ull);
+      return;
+    }
+    if (nbits) {
+      mark(v, nd);
       return;
     }
     const uint32_t old = atomicMin(dist + v, nd);
@@ -168,6 +183,12 @@ struct SsspOp {
         if (c) atomicAdd(nimp, c);
         if (rem) atomicAdd(xops, (unsigned long long)rem);
       }
+      return;
+    }
+    if (nbits) {
+#pragma unroll
+      for (int j = 0; j < K; ++j)
+        if (nd[j] < dv[j]) mark(vv[j], nd[j]);
       return;
     }
 #pragma unroll
@@ -312,8 +333,10 @@ struct SsspDyn {
   SsspDev *s;  // nullptr: static (host-driven) launch
   int32_t *buf[2];
   int32_t *far[2];
-  uint32_t *inq[2];  // claim bitmaps of even / odd iterations
-  uint32_t *keep;    // in-far-pile bitmap
+  uint32_t *inq[2];  // claim bitmaps of even / odd iterations (bitmap mode: frontier C / next N by par)
+  uint32_t *keep;    // in-far-pile bitmap (bitmap mode: the far pile itself)
+  bool bits;         // bitmap frontier (k_sssp_bcompact / k_sssp_bsplit / k_sssp_bpost)
+  int64_t nwords4;   // bitmap mode: words per bitmap, a multiple of 4 (uint4 scans)
 };
 
 __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) { return a > 0xFFFFFFFFu - b ? 0xFFFFFFFFu : a + b; }
@@ -360,6 +383,15 @@ __device__ __forceinline__ bool dyn_bind<SsspOp>(ExpandArgs &a, SsspOp &op, uint
   const bool split = s.nF == 0;
   const int nF = split ? s.nsplit : s.nF;
   if (nF == 0) return false;
+  if (a.dyn.bits) {  // worklist built by k_sssp_bcompact (or the split) in buf[0]
+    a.nF = nF;
+    a.F = a.dyn.buf[0];
+    a.gcount = &a.dyn.s->gcount;
+    op.thr = split ? sat_add(s.thr, s.delta) : s.thr;
+    op.nbits = a.dyn.inq[s.par ^ 1];
+    op.fbits = a.dyn.keep;
+    return true;
+  }
   const int par = s.par, fpar = s.fpar, it = s.iter;
   a.nF = nF;
   a.F = a.dyn.buf[par];
@@ -704,6 +736,105 @@ __global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) {
       if (d >= lo) push(dy.buf[par], &dy.s->nsplit, v);
     }
   }
+}
+
+// ---- bitmap-frontier step (one GPU, CUDA-graph loop) -------------------------------------
+// Step: k_sssp_bcompact (frontier bitmap C -> worklist, C zeroed) -> k_sssp_bsplit (C was
+// empty: far bitmap -> worklist for [thr, thr + delta)) -> k_expand_flat / k_expand_grid
+// (improvements set bits in N = the other bitmap, or in the far bitmap) -> k_sssp_bpost
+// (N becomes C).  The worklist is in vertex order within each CTA's word range.
+constexpr int kCompactNT = 256;
+
+// C -> buf[0] (count in s->nF), C zeroed; one counter atomic per CTA.
+__global__ void __launch_bounds__(kCompactNT) k_sssp_bcompact(SsspDyn dy) {
+  __shared__ __align__(16) SsspDev st_s;
+  load_state(dy.s, &st_s);
+  if (st_s.done) return;
+  using Scan = cub::BlockScan<int, kCompactNT>;
+  __shared__ typename Scan::TempStorage tmp;
+  __shared__ int base_s;
+  uint4 *C = reinterpret_cast<uint4 *>(dy.inq[st_s.par]);
+  int32_t *F = dy.buf[0];
+  const int64_t nv = dy.nwords4 / 4;  // uint4 vectors
+  for (int64_t c0 = (int64_t)blockIdx.x * kCompactNT; c0 < nv; c0 += (int64_t)gridDim.x * kCompactNT) {
+    const int64_t i = c0 + threadIdx.x;
+    uint4 w = make_uint4(0, 0, 0, 0);
+    if (i < nv) w = C[i];
+    const int cnt = __popc(w.x) + __popc(w.y) + __popc(w.z) + __popc(w.w);
+    int off, tot;
+    Scan(tmp).ExclusiveSum(cnt, off, tot);
+    if (threadIdx.x == 0) base_s = tot ? atomicAdd(&dy.s->nF, tot) : 0;
+    __syncthreads();
+    if (cnt) {
+      int pos = base_s + off;
+      const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        for (uint32_t b = ws[q]; b; b &= b - 1) F[pos++] = (int32_t)((i * 4 + q) * 32 + __ffs(b) - 1);
+      C[i] = make_uint4(0, 0, 0, 0);
+    }
+    __syncthreads();  // tmp / base_s reuse
+  }
+}
+
+// Near frontier empty: the far bitmap's vertices with thr <= dist < thr + delta -> buf[0]
+// (count in s->nsplit), those with dist < thr (settled at a smaller distance) dropped, the
+// rest kept (count in s->nfar).
+__global__ void __launch_bounds__(kCompactNT) k_sssp_bsplit(SsspDyn dy, const uint32_t *__restrict__ dist) {
+  __shared__ __align__(16) SsspDev st_s;
+  load_state(dy.s, &st_s);
+  const SsspDev *s = &st_s;
+  if (s->done || s->nF != 0) return;
+  const uint32_t lo = s->thr, hi = sat_add(lo, s->delta);
+  uint4 *Fb = reinterpret_cast<uint4 *>(dy.keep);
+  const int64_t nv = dy.nwords4 / 4;
+  int kept = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nv; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint4 w = Fb[i];
+    if (!(w.x | w.y | w.z | w.w)) continue;
+    uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint32_t keepw = 0;
+      for (uint32_t b = ws[q]; b; b &= b - 1) {
+        const int bit = __ffs(b) - 1;
+        const int32_t v = (int32_t)((i * 4 + q) * 32 + bit);
+        const uint32_t d = dist[v];
+        if (d >= hi) keepw |= 1u << bit;
+        else if (d >= lo) push(dy.buf[0], &dy.s->nsplit, v);
+      }
+      ws[q] = keepw;
+      kept += __popc(keepw);
+    }
+    Fb[i] = make_uint4(ws[0], ws[1], ws[2], ws[3]);
+  }
+  for (int o = 16; o > 0; o >>= 1) kept += __shfl_xor_sync(0xffffffffu, kept, o);
+  if ((threadIdx.x & 31) == 0 && kept) atomicAdd(&dy.s->nfar, kept);
+}
+
+// Roll over: N becomes C; a split step that moved nothing with nothing kept ends the loop.
+__global__ void k_sssp_bpost(SsspDyn dy, cudaGraphConditionalHandle cond, int use_cond) {
+  SsspDev *s = dy.s;
+  if (!s->done) {
+    if (++s->pad > (1 << 20)) s->done = 2;
+    const bool split = s->nF == 0;
+    if (split && s->nsplit == 0 && s->nfar == 0) s->done = 1;
+    if (!s->done) {
+      if (split) s->thr = sat_add(s->thr, s->delta);
+      const int size = split ? s->nsplit : s->nF;
+      if (size > 0) {
+        s->ftotal += (unsigned long long)size;
+        s->iter += 1;
+      }
+      s->par ^= 1;
+      s->nF = 0;
+      s->nsplit = 0;
+      s->nfar = 0;
+      s->gcount = 0;
+      s->slice = 0;
+    }
+  }
+  if (use_cond) cudaGraphSetConditional(cond, s->done ? 0u : 1u);
 }
 
 // Device-driven step, part 4: roll the state over to the next step.  In the CUDA-graph loop
@@ -1248,12 +1379,15 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   const int64_t n = G.n_global;
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
-  const int64_t nwb = (n + 31) / 32 + 1;
-  SsspDyn dy;
+  const int bmode = 0;  // the polling loop keeps the queue-counter worklists
+  const int64_t nwb = ((n + 31) / 32 + 1 + 3) / 4 * 4;  // a multiple of 4 words (uint4 scans)
+  SsspDyn dy{};
   uint32_t *bits = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 3 * nwb);
   dy.inq[0] = bits;
   dy.inq[1] = bits + nwb;
   dy.keep = bits + 2 * nwb;
+  dy.bits = bmode != 0;
+  dy.nwords4 = nwb;
   INL_CUDA(cudaMemsetAsync(bits, 0, sizeof(uint32_t) * 3 * nwb, st));
   dy.far[0] = (int32_t *)ctx->s_g.get(sizeof(int32_t) * (2 * n + 16));
   dy.far[1] = dy.far[0] + n + 8;
@@ -1263,11 +1397,19 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   static_assert(sizeof(SsspDev) <= 64, "SsspDev is read back through the ctx's 64-B pinned buffer");
   const bool owned = source >= G.row_begin && source < G.row_begin + G.n_rows;
   SsspDev h{};
-  h.nF = owned ? 1 : 0;
+  h.nF = owned && !dy.bits ? 1 : 0;
   h.thr = h.delta = sssp_delta();
   INL_CUDA(cudaMemcpyAsync(dy.s, &h, sizeof h, cudaMemcpyHostToDevice, st));
   const int32_t s0 = (int32_t)(owned ? source - G.row_begin : 0);
-  INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  if (dy.bits) {  // the source's bit in C = inq[0]
+    if (owned) {
+      uint32_t *hw = (uint32_t *)ctx->pinned;
+      hw[0] = 1u << (s0 & 31);
+      INL_CUDA(cudaMemcpyAsync(dy.inq[0] + (s0 >> 5), hw, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+    }
+  } else {
+    INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  }
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(dist, n, source);
   INL_CUDA(cudaGetLastError());
   const ExpandCfg c = expand_cfg(G, b);
@@ -1337,6 +1479,7 @@ struct SsspGraphKey {
   int64_t n, nnz, gcap;
   int t_warp, chunk, gm0, gm1, gm2;
   uint32_t delta;
+  int bits;
   bool operator==(const SsspGraphKey &o) const { return memcmp(this, &o, sizeof(*this)) == 0; }
 };
 
@@ -1358,12 +1501,17 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   const int64_t n = G.n_global;
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
-  const int64_t nwb = (n + 31) / 32 + 1;
-  SsspDyn dy;
+  // bitmap frontier by default (INL_SSSP_FRONTIER=list: the r02 queue-counter worklists)
+  const char *fe = getenv("INL_SSSP_FRONTIER");
+  const int bmode = !(fe && !strcmp(fe, "list"));
+  const int64_t nwb = ((n + 31) / 32 + 1 + 3) / 4 * 4;  // a multiple of 4 words (uint4 scans)
+  SsspDyn dy{};
   uint32_t *bits = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 3 * nwb);
   dy.inq[0] = bits;
   dy.inq[1] = bits + nwb;
   dy.keep = bits + 2 * nwb;
+  dy.bits = bmode != 0;
+  dy.nwords4 = nwb;
   INL_CUDA(cudaMemsetAsync(bits, 0, sizeof(uint32_t) * 3 * nwb, st));
   dy.far[0] = (int32_t *)ctx->s_g.get(sizeof(int32_t) * (2 * n + 16));
   dy.far[1] = dy.far[0] + n + 8;
@@ -1372,11 +1520,19 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   dy.s = (SsspDev *)ctx->s_e.get(sizeof(SsspDev));
   const bool owned = source >= G.row_begin && source < G.row_begin + G.n_rows;
   SsspDev h{};
-  h.nF = owned ? 1 : 0;
+  h.nF = owned && !dy.bits ? 1 : 0;
   h.thr = h.delta = sssp_delta();
   INL_CUDA(cudaMemcpyAsync(dy.s, &h, sizeof h, cudaMemcpyHostToDevice, st));
   const int32_t s0 = (int32_t)(owned ? source - G.row_begin : 0);
-  INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  if (dy.bits) {  // the source's bit in C = inq[0]
+    if (owned) {
+      uint32_t *hw = (uint32_t *)ctx->pinned;
+      hw[0] = 1u << (s0 & 31);
+      INL_CUDA(cudaMemcpyAsync(dy.inq[0] + (s0 >> 5), hw, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+    }
+  } else {
+    INL_CUDA(cudaMemcpyAsync(f.F, &s0, sizeof(int32_t), cudaMemcpyHostToDevice, st));
+  }
   k_init_sssp<<<grid_for(n, ctx->num_sms), 256, 0, st>>>(dist, n, source);
   INL_CUDA(cudaGetLastError());
   const ExpandCfg c = expand_cfg(G, b);
@@ -1406,6 +1562,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   key.gm1 = gm[1];
   key.gm2 = gm[2];
   key.delta = h.delta;
+  key.bits = dy.bits;
   SsspGraph *sg = static_cast<SsspGraph *>(ctx->sssp_graph);
   if (!sg || !(sg->key == key)) {
     delete sg;
@@ -1429,10 +1586,20 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     cudaError_t ce = cudaStreamBeginCaptureToGraph(cap, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal);
     if (ce == cudaSuccess) {
       const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
-      k_sssp_split<<<gsplit, 256, 0, cap>>>(dy, dist);
-      k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
-      k_expand_grid<SsspOp><<<ggrid, NT, 0, cap>>>(a, op);
-      k_sssp_post<<<1, 1, 0, cap>>>(dy, cond, 1);
+      if (dy.bits) {
+        const int64_t nv = nwb / 4;
+        int gc = (int)std::min<int64_t>((nv + kCompactNT - 1) / kCompactNT, (int64_t)ctx->num_sms * 8);
+        k_sssp_bcompact<<<gc < 1 ? 1 : gc, kCompactNT, 0, cap>>>(dy);
+        k_sssp_bsplit<<<gc < 1 ? 1 : gc, kCompactNT, 0, cap>>>(dy, dist);
+        k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
+        k_expand_grid<SsspOp><<<ggrid, NT, 0, cap>>>(a, op);
+        k_sssp_bpost<<<1, 1, 0, cap>>>(dy, cond, 1);
+      } else {
+        k_sssp_split<<<gsplit, 256, 0, cap>>>(dy, dist);
+        k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
+        k_expand_grid<SsspOp><<<ggrid, NT, 0, cap>>>(a, op);
+        k_sssp_post<<<1, 1, 0, cap>>>(dy, cond, 1);
+      }
       cudaGraph_t captured = nullptr;
       ce = cudaStreamEndCapture(cap, &captured);
     }
@@ -1461,7 +1628,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
     stats->iterations = hs->iter;
     stats->edges_relaxed = (int64_t)r;
     stats->frontier_total = (int64_t)hs->ftotal;
-    stats->launches = 1 + 4LL * hs->pad;  // init + 4 kernels per step (one graph launch)
+    stats->launches = 1 + (dy.bits ? 5LL : 4LL) * hs->pad;  // init + 4 or 5 kernels per step (one graph launch)
     stats->host_syncs = 1;
     stats->exchange_bytes = 0;
   }

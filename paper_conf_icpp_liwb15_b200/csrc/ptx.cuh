@@ -35,6 +35,14 @@ __device__ __forceinline__ uint32_t ld_stream_pol(const void *p, uint64_t pol) {
   return r;
 }
 
+// fire-and-forget global reductions (RED: the issuing warp never waits for a result)
+__device__ __forceinline__ void red_min_u32(uint32_t *p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.min.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_or_b32(uint32_t *p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
 __device__ __forceinline__ uint64_t policy_evict_last() {
   uint64_t p;
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));

@@ -87,10 +87,14 @@ def test_small_graph_edge_cases(ctx):
         assert np.array_equal(lv, oracle.bfs(rp, ci, s))
 
 
-@pytest.mark.parametrize("loop", ["graph", "dyn"])
+@pytest.mark.parametrize("loop", ["graph", "graph-list", "dyn"])
 def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch):
-    """The device-driven near-far loop: one CUDA-graph launch per source (default) or
-    stream launches with host polling (INL_SSSP_LOOP=dyn), vs the host-driven loop."""
+    """The device-driven near-far loop: one CUDA-graph launch per source (default: bitmap
+    frontier; graph-list: the queue-counter worklists, INL_SSSP_FRONTIER=list) or stream
+    launches with host polling (INL_SSSP_LOOP=dyn), vs the host-driven loop."""
+    if loop == "graph-list":
+        monkeypatch.setenv("INL_SSSP_FRONTIER", "list")
+        loop = "graph"
     monkeypatch.setenv("INL_SSSP_LOOP", loop)
     b = inl.bins(flags=inl.BINS_SSSP_DEVLOOP)
     rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3), (3, 1)], [5, 6, 7], symmetric=True)
