@@ -42,9 +42,12 @@ namespace {
 
 constexpr int NT = 256;
 constexpr int NW = NT / 32;
-// resident CTAs per SM the expansion kernels are compiled for (register cap 65536 / (NT * it))
+// resident CTAs per SM the expansion kernels are compiled for (register cap 65536 / (NT * it)):
+// 4 (64 registers, 32 warps / SM) measured best with the bitmap SSSP loop (scale 23: 4.94 ->
+// 4.48 ms per source; 3: 4.62, 5 and 6 spill: 4.90 / 5.43) and neutral for BFS
+// (profiles/r02/sssp_bitmap_sweeps.txt)
 #ifndef INL_EXPAND_MINB
-#define INL_EXPAND_MINB 1
+#define INL_EXPAND_MINB 4
 #endif
 
 __device__ __forceinline__ void push(int32_t *q, int *cnt, int32_t v) {
@@ -106,6 +109,7 @@ struct SsspOp {
   // expanded with its true distance then), never loses an improvement.
   uint32_t *nbits = nullptr;
   uint32_t *fbits = nullptr;
+  unsigned long long *tmark = nullptr;  // INL_SSSP_TRACE only: improvements marked
   __device__ __forceinline__ void mark(int32_t v, uint32_t nd) const {
     red_min_u32(dist + v, nd);
     red_or_b32((nd >= thr ? fbits : nbits) + (v >> 5), 1u << (v & 31));
@@ -186,9 +190,17 @@ struct SsspOp {
       return;
     }
     if (nbits) {
+      unsigned m = 0;
 #pragma unroll
       for (int j = 0; j < K; ++j)
-        if (nd[j] < dv[j]) mark(vv[j], nd[j]);
+        if (nd[j] < dv[j]) {
+          mark(vv[j], nd[j]);
+          ++m;
+        }
+      if (tmark) {
+        m = __reduce_add_sync(0xffffffffu, m);
+        if ((threadIdx.x & 31) == 0 && m) atomicAdd(tmark, (unsigned long long)m);
+      }
       return;
     }
 #pragma unroll
@@ -339,6 +351,12 @@ struct SsspDyn {
   int64_t nwords4;   // bitmap mode: words per bitmap, a multiple of 4 (uint4 scans)
 };
 
+// element i & 1 of a two-entry array held in a kernel parameter, without indexing it: a
+// run-time index forces the whole parameter struct into a per-thread stack copy (~200 B of
+// local stores per thread at kernel entry, ~10 us per launch of an otherwise idle grid)
+template <class T>
+__device__ __forceinline__ T pick2(T const (&v)[2], int i) { return (i & 1) ? v[1] : v[0]; }
+
 __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) { return a > 0xFFFFFFFFu - b ? 0xFFFFFFFFu : a + b; }
 
 struct ExpandArgs {
@@ -388,22 +406,66 @@ __device__ __forceinline__ bool dyn_bind<SsspOp>(ExpandArgs &a, SsspOp &op, uint
     a.F = a.dyn.buf[0];
     a.gcount = &a.dyn.s->gcount;
     op.thr = split ? sat_add(s.thr, s.delta) : s.thr;
-    op.nbits = a.dyn.inq[s.par ^ 1];
+    op.nbits = pick2(a.dyn.inq, s.par ^ 1);
     op.fbits = a.dyn.keep;
     return true;
   }
   const int par = s.par, fpar = s.fpar, it = s.iter;
   a.nF = nF;
-  a.F = a.dyn.buf[par];
-  a.Fout = a.dyn.buf[par ^ 1];
+  a.F = pick2(a.dyn.buf, par);
+  a.Fout = pick2(a.dyn.buf, par ^ 1);
   a.fcount = &a.dyn.s->cnt;
   a.gcount = &a.dyn.s->gcount;
   op.thr = split ? sat_add(s.thr, s.delta) : s.thr;
-  op.inq = a.dyn.inq[it & 1];
-  op.far = a.dyn.far[split ? fpar ^ 1 : fpar];
+  op.inq = pick2(a.dyn.inq, it & 1);
+  op.far = pick2(a.dyn.far, split ? fpar ^ 1 : fpar);
   op.far_count = split ? &a.dyn.s->nfar2 : &a.dyn.s->nfar;
   op.infar = a.dyn.keep;
-  *inq_prev = a.dyn.inq[(it & 1) ^ 1];
+  *inq_prev = pick2(a.dyn.inq, (it & 1) ^ 1);
+  return true;
+}
+
+// The bitmap graph loop's relaxation alone (SsspOp::edges minus the NEXT-1 and worklist
+// paths): the expansion kernels instantiated for it carry no registers for the paths they never
+// take (64 registers without spills at 4 resident CTAs / SM; SsspOp spills ~200 B there).
+struct SsspBitsOp : SsspOp {
+  template <int K>
+  __device__ __forceinline__ void edges(const uint32_t (&du)[K], const int64_t (&kk)[K], const int32_t (&vv)[K],
+                                        const bool (&in)[K], int32_t *, int *) const {
+    uint32_t nd[K], dv[K];
+#pragma unroll
+    for (int j = 0; j < K; ++j) nd[j] = in[j] ? du[j] + ld_stream_pol(w + kk[j], pol_stream) : 0xFFFFFFFFu;
+#pragma unroll
+    for (int j = 0; j < K; ++j) dv[j] = in[j] ? dist[vv[j]] : 0u;
+    unsigned m = 0;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (nd[j] < dv[j]) {
+        mark(vv[j], nd[j]);
+        ++m;
+      }
+    if (tmark) {
+      m = __reduce_add_sync(0xffffffffu, m);
+      if ((threadIdx.x & 31) == 0 && m) atomicAdd(tmark, (unsigned long long)m);
+    }
+  }
+};
+template <>
+__device__ __forceinline__ bool dyn_bind<SsspBitsOp>(ExpandArgs &a, SsspBitsOp &op, uint32_t **inq_prev) {
+  *inq_prev = nullptr;
+  __shared__ __align__(16) SsspDev st_s;
+  load_state(a.dyn.s, &st_s);
+  const SsspDev &s = st_s;
+  if (s.done) return false;
+  const bool split = s.nF == 0;
+  const int nF = split ? s.nsplit : s.nF;
+  if (nF == 0) return false;
+  a.nF = nF;  // worklist built by k_sssp_bcompact (or the split) in buf[0]
+  a.F = a.dyn.buf[0];
+  a.gcount = &a.dyn.s->gcount;
+  op.thr = split ? sat_add(s.thr, s.delta) : s.thr;
+  op.nbits = pick2(a.dyn.inq, s.par ^ 1);
+  op.fbits = a.dyn.keep;
   return true;
 }
 
@@ -535,6 +597,10 @@ constexpr int kEdgesPerThread = 8;
 
 template <class Op>
 __global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs a, Op op) {
+  if (a.dyn.s) {  // device-sized step: CTAs beyond the frontier's slices leave before any setup
+    const int nf = __ldcg(&a.dyn.s->nF);
+    if ((int64_t)blockIdx.x * NT >= (nf ? nf : __ldcg(&a.dyn.s->nsplit))) return;
+  }
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
@@ -645,6 +711,8 @@ __global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs 
 // frontier vertices, one CTA per piece (grid-stride); each thread keeps 8 edges in flight.
 template <class Op>
 __global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_grid(ExpandArgs a, Op op) {
+  // device-sized step: CTAs beyond the pieces the flat kernel emitted leave before any setup
+  if (a.dyn.s && blockIdx.x >= min(__ldcg(&a.dyn.s->gcount), a.gcap)) return;
   op.pol_stream = policy_evict_first();
   uint32_t *inq_prev;
   if (!dyn_bind(a, op, &inq_prev)) return;
@@ -725,15 +793,15 @@ __global__ void k_sssp_split(SsspDyn dy, const uint32_t *__restrict__ dist) {
   }
   const uint32_t lo = s->thr, hi = sat_add(lo, s->delta);
   const int fpar = s->fpar, par = s->par;
-  const int32_t *far = dy.far[fpar];
+  const int32_t *far = pick2(dy.far, fpar);
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < nfar; i += gridDim.x * blockDim.x) {
     const int32_t v = far[i];
     const uint32_t d = dist[v];
     if (d >= hi) {
-      push(dy.far[fpar ^ 1], &dy.s->nfar2, v);
+      push(pick2(dy.far, fpar ^ 1), &dy.s->nfar2, v);
     } else {
       atomicAnd(dy.keep + (v >> 5), ~(1u << (v & 31)));
-      if (d >= lo) push(dy.buf[par], &dy.s->nsplit, v);
+      if (d >= lo) push(pick2(dy.buf, par), &dy.s->nsplit, v);
     }
   }
 }
@@ -753,7 +821,7 @@ __global__ void __launch_bounds__(kCompactNT) k_sssp_bcompact(SsspDyn dy) {
   using Scan = cub::BlockScan<int, kCompactNT>;
   __shared__ typename Scan::TempStorage tmp;
   __shared__ int base_s;
-  uint4 *C = reinterpret_cast<uint4 *>(dy.inq[st_s.par]);
+  uint4 *C = reinterpret_cast<uint4 *>(pick2(dy.inq, st_s.par));
   int32_t *F = dy.buf[0];
   const int64_t nv = dy.nwords4 / 4;  // uint4 vectors
   for (int64_t c0 = (int64_t)blockIdx.x * kCompactNT; c0 < nv; c0 += (int64_t)gridDim.x * kCompactNT) {
@@ -835,6 +903,25 @@ __global__ void k_sssp_bpost(SsspDyn dy, cudaGraphConditionalHandle cond, int us
     }
   }
   if (use_cond) cudaGraphSetConditional(cond, s->done ? 0u : 1u);
+}
+
+// INL_SSSP_TRACE=<file> (measurement only): a one-thread kernel between the step kernels of the
+// bitmap graph loop stamps %globaltimer, so the host can print each step's kernel durations and
+// frontier sizes.  slot 0..5: step start, after compact, split, flat, grid, post; 6: nF | nsplit.
+constexpr int kTraceSlots = 12, kTraceSteps = 4096;
+__global__ void k_sssp_trace(const SsspDev *s, unsigned long long *tr, int slot, const unsigned long long *relaxed,
+                             const unsigned long long *marks) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  const int step = s->pad;
+  if (step >= kTraceSteps) return;
+  unsigned long long *r = tr + step * kTraceSlots;
+  r[slot] = t;
+  if (slot == 3) r[6] = (unsigned long long)(unsigned)s->nF | ((unsigned long long)(unsigned)s->nsplit << 32);
+  if (slot == 3 || slot == 4) {  // 7 / 8: relaxed / marked after the flat kernel; 9 / 10 after the grid kernel
+    r[slot == 3 ? 7 : 9] = *relaxed;
+    r[slot == 3 ? 8 : 10] = marks ? *marks : 0ull;
+  }
 }
 
 // Device-driven step, part 4: roll the state over to the next step.  In the CUDA-graph loop
@@ -1237,7 +1324,10 @@ int grid_for(int64_t n, int sms) {
 uint32_t sssp_delta() {
   static uint32_t d = 0;
   if (!d) {
-    d = 48;  // measured best on R-MAT scale 23, w in [1, 255] (profiles/r01/sssp_delta_sweep2.txt)
+    // near-far delta on R-MAT scale 23, w in [1, 255]: 48 with the round-1 worklists
+    // (profiles/r01/sssp_delta_sweep2.txt); 96 with the bitmap loop at 32 warps / SM (4.33 ->
+    // 4.03 ms; 128..384 within 2% but more wasted relaxations; profiles/r02/sssp_bitmap_sweeps.txt)
+    d = 96;
     if (const char *e = getenv("INL_SSSP_DELTA")) d = (uint32_t)strtoul(e, nullptr, 10);
     if (!d) d = 0xFFFFFFFFu;
   }
@@ -1379,7 +1469,11 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   const int64_t n = G.n_global;
   FrontierBufs f = frontier_bufs(ctx, G, b);
   INL_CUDA(cudaMemsetAsync(f.relaxed, 0, sizeof(unsigned long long), st));
-  const int bmode = 0;  // the polling loop keeps the queue-counter worklists
+  // the polling loop keeps the queue-counter worklists; INL_SSSP_DYN_BITS=1 runs the graph loop's
+  // bitmap step kernels stream-launched instead (so ncu can profile them: it skips kernels inside
+  // conditional graph nodes)
+  const char *dbe = getenv("INL_SSSP_DYN_BITS");
+  const int bmode = dbe && atoi(dbe) != 0;
   const int64_t nwb = ((n + 31) / 32 + 1 + 3) / 4 * 4;  // a multiple of 4 words (uint4 scans)
   SsspDyn dy{};
   uint32_t *bits = (uint32_t *)ctx->s_d.get(sizeof(uint32_t) * 3 * nwb);
@@ -1421,14 +1515,33 @@ static void sssp_run_dyn(inl_ctx ctx, const inl_csr &G, const Bins &b, const uin
   static int gm[3] = {2, 8, 2};
   if (gmul < 0) {
     gmul = 1;
+    if (bmode) gm[1] = 6, gm[2] = 8;  // the graph loop's bitmap-step grids
     if (const char *e = getenv("INL_SSSP_GRIDS")) sscanf(e, "%d,%d,%d", &gm[0], &gm[1], &gm[2]);
   }
   const int gsplit = ctx->num_sms * gm[0], gflat = ctx->num_sms * gm[1], ggrid = ctx->num_sms * gm[2];
+  SsspBitsOp bop;
+  static_cast<SsspOp &>(bop) = op;
+  const int64_t nv4 = nwb / 4;
+  const int gc = (int)std::max<int64_t>(1, std::min<int64_t>((nv4 + kCompactNT - 1) / kCompactNT, (int64_t)ctx->num_sms * 8));
   int64_t launches = 1, syncs = 0;
   int batch = 4;
   SsspDev *hs = (SsspDev *)ctx->pinned;  // pinned scratch (>= 64 B)
   for (;;) {
-    for (int k = 0; k < batch; ++k) {
+    for (int k = 0; k < batch && bmode; ++k) {
+      k_sssp_bcompact<<<gc, kCompactNT, 0, st>>>(dy);
+      k_sssp_bsplit<<<gc, kCompactNT, 0, st>>>(dy, dist);
+      {
+        KScope ks(ctx, "k_expand_flat");
+        k_expand_flat<SsspBitsOp><<<gflat, NT, 0, st>>>(a, bop);
+      }
+      {
+        KScope ks(ctx, "k_expand_grid");
+        k_expand_grid<SsspBitsOp><<<ggrid, NT, 0, st>>>(a, bop);
+      }
+      k_sssp_bpost<<<1, 1, 0, st>>>(dy, 0, 0);
+      launches += 5;
+    }
+    for (int k = 0; k < batch && !bmode; ++k) {
       {
         KScope ks(ctx, "k_sssp_split");
         k_sssp_split<<<gsplit, 256, 0, st>>>(dy, dist);
@@ -1480,6 +1593,7 @@ struct SsspGraphKey {
   int t_warp, chunk, gm0, gm1, gm2;
   uint32_t delta;
   int bits;
+  void *trace;
   bool operator==(const SsspGraphKey &o) const { return memcmp(this, &o, sizeof(*this)) == 0; }
 };
 
@@ -1540,7 +1654,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
                f.gitems, nullptr, (int)f.gcap, f.counts + 2, f.Fout, nullptr, f.relaxed};
   a.dyn = dy;
   SsspOp op{dist, w, nullptr, nullptr, 0, 0, true, 0, 0, nullptr, nullptr, nullptr};
-  static int gm[3] = {2, 8, 2};
+  static int gm[3] = {2, 6, 8};  // split, flat, grid CTAs per SM (sweep: profiles/r02/sssp_bitmap_sweeps.txt)
   static bool gm_read = false;
   if (!gm_read) {
     gm_read = true;
@@ -1563,6 +1677,16 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   key.gm2 = gm[2];
   key.delta = h.delta;
   key.bits = dy.bits;
+  const char *trace_path = getenv("INL_SSSP_TRACE");
+  unsigned long long *trace = nullptr;
+  if (trace_path && dy.bits) {
+    trace = (unsigned long long *)ctx->s_t.get(sizeof(unsigned long long) * (kTraceSlots * kTraceSteps + 1));
+    INL_CUDA(cudaMemsetAsync(trace, 0, sizeof(unsigned long long) * (kTraceSlots * kTraceSteps + 1), st));
+    // the improvement counter (one same-address atomic per warp-call) slows the step kernels
+    // severalfold, so it is on only with INL_SSSP_TRACE_MARKS (counts from one run, times from another)
+    if (getenv("INL_SSSP_TRACE_MARKS")) op.tmark = trace + kTraceSlots * kTraceSteps;
+  }
+  key.trace = trace;
   SsspGraph *sg = static_cast<SsspGraph *>(ctx->sssp_graph);
   if (!sg || !(sg->key == key)) {
     delete sg;
@@ -1589,11 +1713,22 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
       if (dy.bits) {
         const int64_t nv = nwb / 4;
         int gc = (int)std::min<int64_t>((nv + kCompactNT - 1) / kCompactNT, (int64_t)ctx->num_sms * 8);
+        auto tr = [&](int slot) {
+          if (trace) k_sssp_trace<<<1, 1, 0, cap>>>(dy.s, trace, slot, f.relaxed, op.tmark);
+        };
+        tr(0);
         k_sssp_bcompact<<<gc < 1 ? 1 : gc, kCompactNT, 0, cap>>>(dy);
+        tr(1);
         k_sssp_bsplit<<<gc < 1 ? 1 : gc, kCompactNT, 0, cap>>>(dy, dist);
-        k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
-        k_expand_grid<SsspOp><<<ggrid, NT, 0, cap>>>(a, op);
+        tr(2);
+        SsspBitsOp bop;
+        static_cast<SsspOp &>(bop) = op;
+        k_expand_flat<SsspBitsOp><<<gflat, NT, 0, cap>>>(a, bop);
+        tr(3);
+        k_expand_grid<SsspBitsOp><<<ggrid, NT, 0, cap>>>(a, bop);
+        tr(4);
         k_sssp_bpost<<<1, 1, 0, cap>>>(dy, cond, 1);
+        tr(5);
       } else {
         k_sssp_split<<<gsplit, 256, 0, cap>>>(dy, dist);
         k_expand_flat<SsspOp><<<gflat, NT, 0, cap>>>(a, op);
@@ -1620,6 +1755,23 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
   ctx_sync(ctx);
   if (((volatile SsspDev *)hs)->done == 2)
     raise(INL_ERR_INTERNAL, "sssp graph loop exceeded its step bound");
+  if (trace) {  // measurement only: append this call's per-step trace to the file
+    const int steps = std::min(hs->pad + 1, kTraceSteps);
+    std::vector<unsigned long long> h((size_t)steps * kTraceSlots);
+    INL_CUDA(cudaMemcpy(h.data(), trace, h.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+    if (FILE *fp = fopen(trace_path, "a")) {
+      fprintf(fp, "# source %lld\n", (long long)source);
+      for (int i = 0; i < steps; ++i) {
+        const unsigned long long *r = &h[(size_t)i * kTraceSlots];
+        fprintf(fp, "%d", i);
+        for (int k = 0; k < 6; ++k) fprintf(fp, " %llu", r[k]);
+        fprintf(fp, " %u %u", (unsigned)(r[6] & 0xffffffffu), (unsigned)(r[6] >> 32));
+        for (int k = 7; k < 11; ++k) fprintf(fp, " %llu", r[k]);
+        fprintf(fp, "\n");
+      }
+      fclose(fp);
+    }
+  }
   check_overflow(ctx, f);
   if (stats) {
     unsigned long long r = 0;

@@ -5,6 +5,8 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
+#include <cstdlib>
 #include <vector>
 
 #include "inl.h"
@@ -154,6 +156,7 @@ struct inl_ctx_s {
   inl::DevBuf s_pad;                                   // padded replicated vectors (P > 1)
   inl::DevBuf s_bu;                                    // BFS bottom-up worklists
   inl::DevBuf s_h;                                     // tree levels (tree.cu)
+  inl::DevBuf s_t;                                     // SSSP step trace (INL_SSSP_TRACE, measurement)
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
@@ -229,6 +232,35 @@ struct KScope {
     sl->pending.emplace_back(e0, e1);
   }
 };
+// Whether PDL launches are on (INL_PDL=0 turns them off, for A/B measurement).
+inline bool pdl_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("INL_PDL");
+    v = e ? atoi(e) != 0 : 1;
+  }
+  return v == 1;
+}
+
+// Launch `k` on ctx's stream with a programmatic dependency on the previous kernel of the stream
+// (cudaLaunchAttributeProgrammaticStreamSerialization): its CTAs may launch while that kernel
+// drains, and must call pdl_wait() before touching anything the previous kernel writes or reads.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                       Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
+}
+
 // plan.cu
 void build_plan(inl_plan p);
 // spmv.cu
