@@ -748,7 +748,14 @@ inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level
     StagedOut<int32_t> o = stage_out(ctx->h_y, level, G->n_global);
     Bins b = plan ? plan->bins : resolve_bins(nullptr);
     if (plan) INL_CHECK(plan->ctx == ctx && same_csr(plan, d), "plan was created for a different CSR");
-    bfs_run(ctx, d, b, source, o.dev, stats, plan && plan->symmetric);
+    BuStatic bus;
+    if (plan && plan->symmetric && plan->bu_ns + plan->bu_nl > 0) {
+      bus.s = (const int32_t *)plan->bu_lists.p;
+      bus.l = bus.s + plan->n_global;
+      bus.ns = plan->bu_ns;
+      bus.nl = plan->bu_nl;
+    }
+    bfs_run(ctx, d, b, source, o.dev, stats, plan && plan->symmetric, bus);
     finish_out(ctx, o);
     ctx_sync(ctx);
   });

@@ -1106,6 +1106,14 @@ struct BuBin {  // unvisited, degree in (lo, hi]
     return d > lo && d <= hi;
   }
 };
+struct BuDeg {  // degree in (lo, hi]
+  const int64_t *rp;
+  int64_t lo, hi;
+  __device__ __forceinline__ bool operator()(int32_t v) const {
+    const int64_t d = rp[v + 1] - rp[v];
+    return d > lo && d <= hi;
+  }
+};
 struct BuUnvisited {
   const uint32_t *visited;
   __device__ __forceinline__ bool operator()(int32_t v) const { return !((visited[v >> 5] >> (v & 31)) & 1u); }
@@ -1125,7 +1133,14 @@ struct BuArgs {
   unsigned long long *mf;  // their degree sum (Beamer's m_f)
   uint64_t pol;
   unsigned long long *examined;  // neighbours read (the stats' edges_relaxed)
+  // `in` is the plan's static degree bin (every vertex of degree > 0, visited or not): skip the
+  // visited ones (the first bottom-up level; later levels read the compacted unvisited lists)
+  bool check_visited = false;
 };
+
+__device__ __forceinline__ bool bu_skip(const BuArgs &a, int32_t v) {
+  return a.check_visited && ((__ldg(a.visited + (v >> 5)) >> (v & 31)) & 1u);
+}
 
 __device__ __forceinline__ void bu_visit(const BuArgs &a, int32_t v) {
   const uint32_t bit = 1u << (v & 31);
@@ -1142,8 +1157,9 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
   int fcnt = 0;
   unsigned long long dg = 0, ex = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nn; i += stride) {
-    const bool valid = i < a.n_in;
+    bool valid = i < a.n_in;
     const int32_t v = valid ? a.in[i] : 0;
+    if (valid && bu_skip(a, v)) valid = false;
     bool found = false;
     int64_t s = 0, e = 0;
     if (valid) {
@@ -1205,8 +1221,9 @@ __global__ void __launch_bounds__(256) k_bu_group(BuArgs a, int32_t *deep, int *
   int fcnt = 0;
   unsigned long long dg = 0, ex = 0;
   for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / G; i < nn; i += ngroups) {
-    const bool valid = i < a.n_in;
+    bool valid = i < a.n_in;
     const int32_t v = valid ? a.in[i] : 0;
+    if (valid && bu_skip(a, v)) valid = false;
     int64_t s = 0, e = 0;
     if (valid) {
       s = a.rp[v];
@@ -1954,8 +1971,33 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
   finish_stats(ctx, f, stats, iters, ftotal, xbytes);
 }
 
+// The plan's static bottom-up bins (a3's degree binning applied to the bottom-up loop): every
+// vertex of degree in (0, kBuThread] (thread bin), then every vertex of larger degree (warp bin),
+// each in vertex order.  The first bottom-up level of a BFS reads them (skipping visited
+// vertices) instead of partitioning all n vertices on the device at that level.
+void bu_static_build(inl_plan p) {
+  inl_ctx ctx = p->ctx;
+  cudaStream_t st = ctx->stream;
+  const int64_t n = p->n_global;
+  p->bu_ns = p->bu_nl = 0;
+  if (n < 4096 || n > INT32_MAX - 1) return;  // BFS takes bottom-up steps only from n >= 4096
+  int32_t *lists = (int32_t *)p->bu_lists.get(sizeof(int32_t) * 2 * (size_t)n);
+  int *cnt = (int *)ctx->s_f.get(64);
+  thrust::counting_iterator<int32_t> iota(0);
+  thrust::discard_iterator<> none;
+  const BuDeg sm{p->row_ptr, 0, kBuThread}, lg{p->row_ptr, kBuThread, INT64_MAX};
+  size_t need = 0;
+  INL_CUDA(cub::DevicePartition::If(nullptr, need, iota, lists, lists + n, none, cnt, (int)n, sm, lg, st));
+  INL_CUDA(cub::DevicePartition::If(ctx->s_tmp.get(need), need, iota, lists, lists + n, none, cnt, (int)n, sm, lg, st));
+  int h[2] = {0, 0};
+  INL_CUDA(cudaMemcpyAsync(h, cnt, sizeof h, cudaMemcpyDeviceToHost, st));
+  INL_CUDA(cudaStreamSynchronize(st));
+  p->bu_ns = h[0];
+  p->bu_nl = h[1];
+}
+
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
-             inl_stats *stats, bool symmetric) {
+             inl_stats *stats, bool symmetric, const BuStatic &bus) {
   cudaStream_t st = ctx->stream;
   const int64_t n = G.n_global;
   const bool DIST = has_comm(ctx);  // row-block mode with an exchange (NCCL or loopback; also P = 1)
@@ -2067,6 +2109,13 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           INL_CUDA(cudaGetLastError());
           read_level(&nF, &mf_next);
         } else {
+          const bool from_static = !lists_ok && bus.s;  // the plan's degree bins, visited ones skipped
+          if (from_static) {
+            n_small = (int)bus.ns;
+            n_large = (int)bus.nl;
+            bl_cur = 0;
+            lists_ok = true;
+          }
           if (!lists_ok) {  // entering bottom-up: the unvisited vertices, binned by degree
             thrust::counting_iterator<int32_t> iota(0);
             size_t need = 0;
@@ -2084,7 +2133,8 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           }
           INL_CUDA(cudaMemsetAsync(fb, 0, sizeof(uint32_t) * nwords, st));
           INL_CUDA(cudaMemsetAsync(f.counts + 6, 0, 2 * sizeof(int), st));
-          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, bl_s[bl_cur], n_small, f.counts, mfp, 0, f.relaxed};
+          const int32_t *in_s = from_static ? bus.s : bl_s[bl_cur], *in_l = from_static ? bus.l : bl_l[bl_cur];
+          BuArgs ba{G.row_ptr, G.col_idx, fa, fb, bm, level, L, in_s, n_small, f.counts, mfp, 0, f.relaxed, from_static};
           if (n_small > 0) {
             if (bu_small_thread) {
               KScope ks(ctx, "k_bu_thread");
@@ -2095,7 +2145,7 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
                                                                                                    nullptr);
             }
           }
-          ba.in = bl_l[bl_cur];
+          ba.in = in_l;
           ba.n_in = n_large;
           if (n_large > 0) {
             int32_t *deep = bl_l[bl_cur ^ 1];  // the next large list is written only after k_bu_deep
@@ -2113,14 +2163,14 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           const BuUnvisited un{bm};
           if (n_small > 0) {
             size_t need = 0;
-            INL_CUDA(cub::DeviceSelect::If(nullptr, need, bl_s[bl_cur], bl_s[bl_cur ^ 1], f.counts + 6, n_small, un, st));
-            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, bl_s[bl_cur], bl_s[bl_cur ^ 1], f.counts + 6,
+            INL_CUDA(cub::DeviceSelect::If(nullptr, need, in_s, bl_s[bl_cur ^ 1], f.counts + 6, n_small, un, st));
+            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, in_s, bl_s[bl_cur ^ 1], f.counts + 6,
                                            n_small, un, st));
           }
           if (n_large > 0) {
             size_t need = 0;
-            INL_CUDA(cub::DeviceSelect::If(nullptr, need, bl_l[bl_cur], bl_l[bl_cur ^ 1], f.counts + 7, n_large, un, st));
-            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, bl_l[bl_cur], bl_l[bl_cur ^ 1], f.counts + 7,
+            INL_CUDA(cub::DeviceSelect::If(nullptr, need, in_l, bl_l[bl_cur ^ 1], f.counts + 7, n_large, un, st));
+            INL_CUDA(cub::DeviceSelect::If(ctx->s_tmp.get(need), need, in_l, bl_l[bl_cur ^ 1], f.counts + 7,
                                            n_large, un, st));
           }
           read_level(&nF, &mf_next);

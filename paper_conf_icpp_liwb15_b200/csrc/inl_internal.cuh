@@ -209,6 +209,10 @@ struct inl_plan_s {
   inl::DevBuf pr_hot;          // int32 [pr_nhot]: hot slots in the compact space
   int64_t pr_nhot = 0;         // PageRank's hot slots (a prefix of the plan's)
   bool symmetric = false;  // every edge's reverse is present (checked at plan time, sorted rows)
+  // static bottom-up bins of a symmetric plan (frontier.cu bu_static_build): thread bin
+  // [0, bu_ns), warp bin [n_global, n_global + bu_nl) of bu_lists
+  inl::DevBuf bu_lists;
+  int64_t bu_ns = 0, bu_nl = 0;
   // column-blocked long rows: SpMV (the CSR's column space) and PageRank (compact space)
   inl::CbPlan cb, pr_cb;
 };
@@ -274,8 +278,13 @@ void sssp_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const uint32_t *w, i
               uint32_t *dist, inl_stats *st);
 // symmetric: the plan verified that every edge (u, v) has its reverse (v, u), so a vertex's
 // row lists its predecessors too (bottom-up / pull steps are valid)
+struct BuStatic {  // a plan's static bottom-up bins (s == nullptr: none)
+  const int32_t *s = nullptr, *l = nullptr;
+  int64_t ns = 0, nl = 0;
+};
 void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32_t *level,
-             inl_stats *st, bool symmetric);
+             inl_stats *st, bool symmetric, const BuStatic &bus = BuStatic());
+void bu_static_build(inl_plan p);
 // templates.cu: the paper's dual-queue / dbuf-global / dbuf-shared SpMV (false: no template flag)
 constexpr int kTemplateFlags = INL_BINS_TPL_DUAL_QUEUE | INL_BINS_TPL_DBUF_GLOBAL | INL_BINS_TPL_DBUF_SHARED;
 bool spmv_template(inl_ctx ctx, const inl_csr &A, const Bins &b, const float *val, const float *x, float *y);

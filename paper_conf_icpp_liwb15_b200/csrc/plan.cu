@@ -381,6 +381,7 @@ void build_plan(inl_plan p) {
     INL_CUDA(cudaMemcpyAsync(&h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
     INL_CUDA(cudaStreamSynchronize(st));
     p->symmetric = h_bad == 0;
+    if (p->symmetric) bu_static_build(p);
   }
   p->info.symmetric = p->symmetric ? 1 : 0;
   cb_build(p, p->cb, p->col_idx, p->n_global);
