@@ -856,25 +856,43 @@ __global__ void __launch_bounds__(kCompactNT) k_sssp_bsplit(SsspDyn dy, const ui
   const uint32_t lo = s->thr, hi = sat_add(lo, s->delta);
   uint4 *Fb = reinterpret_cast<uint4 *>(dy.keep);
   const int64_t nv = dy.nwords4 / 4;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t nvr = (nv + 31) / 32 * 32;  // whole warps iterate together (warp-aggregated pushes)
+  const int lane = threadIdx.x & 31;
   int kept = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nv; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint4 w = Fb[i];
-    if (!(w.x | w.y | w.z | w.w)) continue;
-    uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nvr; i += stride) {
+    const uint4 w = i < nv ? Fb[i] : make_uint4(0, 0, 0, 0);
+    uint32_t ws[4] = {w.x, w.y, w.z, w.w}, pm[4] = {0u, 0u, 0u, 0u};
+    int c = 0;
+    if (w.x | w.y | w.z | w.w) {
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      uint32_t keepw = 0;
-      for (uint32_t b = ws[q]; b; b &= b - 1) {
-        const int bit = __ffs(b) - 1;
-        const int32_t v = (int32_t)((i * 4 + q) * 32 + bit);
-        const uint32_t d = dist[v];
-        if (d >= hi) keepw |= 1u << bit;
-        else if (d >= lo) push(dy.buf[0], &dy.s->nsplit, v);
+      for (int q = 0; q < 4; ++q) {
+        uint32_t keepw = 0;
+        for (uint32_t b = ws[q]; b; b &= b - 1) {
+          const int bit = __ffs(b) - 1;
+          const uint32_t d = dist[(i * 4 + q) * 32 + bit];
+          if (d >= hi) keepw |= 1u << bit;
+          else if (d >= lo) pm[q] |= 1u << bit;
+        }
+        c += __popc(pm[q]);
+        kept += __popc(keepw);
+        ws[q] = keepw;
       }
-      ws[q] = keepw;
-      kept += __popc(keepw);
+      Fb[i] = make_uint4(ws[0], ws[1], ws[2], ws[3]);
     }
-    Fb[i] = make_uint4(ws[0], ws[1], ws[2], ws[3]);
+    if (!__any_sync(0xffffffffu, c != 0)) continue;
+    int incl = c;  // one counter atomic per warp instead of one per moved vertex
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
+    int base = 0;
+    if (lane == 31) base = atomicAdd(&dy.s->nsplit, incl);
+    int pos = __shfl_sync(0xffffffffu, base, 31) + incl - c;
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      for (uint32_t b = pm[q]; b; b &= b - 1) dy.buf[0][pos++] = (int32_t)((i * 4 + q) * 32 + __ffs(b) - 1);
   }
   for (int o = 16; o > 0; o >>= 1) kept += __shfl_xor_sync(0xffffffffu, kept, o);
   if ((threadIdx.x & 31) == 0 && kept) atomicAdd(&dy.s->nfar, kept);
