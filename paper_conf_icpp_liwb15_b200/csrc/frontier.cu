@@ -1168,6 +1168,7 @@ __device__ __forceinline__ void bu_visit(const BuArgs &a, int32_t v) {
 }
 
 // thread bin: one lane per vertex, its <= kBuThread neighbours 8 at a time
+template <int K1>  // neighbours probed in the first batch (then 8 per batch)
 __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
   a.pol = policy_evict_first();
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -1184,7 +1185,21 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
       s = a.rp[v];
       e = a.rp[v + 1];
     }
-    for (int64_t k = s; k < e && !found; k += 8) {
+    int64_t k = s;
+    if (K1 < 8 && k < e) {  // a short first batch: most vertices find a parent among their first neighbours
+      ex += (unsigned long long)min((int64_t)K1, e - k);
+      int32_t u[K1];
+#pragma unroll
+      for (int j = 0; j < K1; ++j) u[j] = k + j < e ? (int32_t)ld_stream_pol(a.col + k + j, a.pol) : -1;
+      uint32_t fw[K1];
+#pragma unroll
+      for (int j = 0; j < K1; ++j) fw[j] = u[j] >= 0 ? __ldg(a.fcur + (u[j] >> 5)) : 0u;
+#pragma unroll
+      for (int j = 0; j < K1; ++j)
+        if (u[j] >= 0 && ((fw[j] >> (u[j] & 31)) & 1u)) found = true;
+      k += K1;
+    }
+    for (; k < e && !found; k += 8) {
       ex += (unsigned long long)min((int64_t)8, e - k);
       int32_t u[8];
 #pragma unroll
@@ -2156,7 +2171,15 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
           if (n_small > 0) {
             if (bu_small_thread) {
               KScope ks(ctx, "k_bu_thread");
-              k_bu_thread<<<grid_for(n_small, ctx->num_sms), 256, 0, st>>>(ba);
+              // first-batch width: 2 (scale 26: 2.70 -> 2.50 ms per BFS; 4: 2.56, 1: 2.52; scale 23
+              // within noise; profiles/r02/bfs_k1_sweep.txt); INL_BFS_K1 = 1 / 2 / 4 / 8 to measure
+              static int k1 = -1;
+              if (k1 < 0) k1 = getenv("INL_BFS_K1") ? atoi(getenv("INL_BFS_K1")) : 2;
+              const int gb = (int)grid_for(n_small, ctx->num_sms);
+              if (k1 == 1) k_bu_thread<1><<<gb, 256, 0, st>>>(ba);
+              else if (k1 == 2) k_bu_thread<2><<<gb, 256, 0, st>>>(ba);
+              else if (k1 == 4) k_bu_thread<4><<<gb, 256, 0, st>>>(ba);
+              else k_bu_thread<8><<<gb, 256, 0, st>>>(ba);
             } else {
               KScope ks(ctx, "k_bu_small");
               k_bu_group<4, kBuThread, false><<<grid_for((int64_t)n_small * 4, ctx->num_sms), 256, 0, st>>>(ba, nullptr,
