@@ -87,14 +87,24 @@ def test_small_graph_edge_cases(ctx):
         assert np.array_equal(lv, oracle.bfs(rp, ci, s))
 
 
-@pytest.mark.parametrize("loop", ["graph", "graph-list", "dyn"])
-def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch):
+@pytest.mark.parametrize("loop", ["graph", "graph-list", "graph-trace", "dyn", "dyn-bits"])
+def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch, tmp_path):
     """The device-driven near-far loop: one CUDA-graph launch per source (default: bitmap
-    frontier; graph-list: the queue-counter worklists, INL_SSSP_FRONTIER=list) or stream
-    launches with host polling (INL_SSSP_LOOP=dyn), vs the host-driven loop."""
+    frontier; graph-list: the queue-counter worklists, INL_SSSP_FRONTIER=list; graph-trace: with
+    the per-step %globaltimer trace and improvement counter) or stream launches with host polling
+    (INL_SSSP_LOOP=dyn; dyn-bits: the graph loop's bitmap step kernels), vs the host-driven loop."""
+    trace = None
     if loop == "graph-list":
         monkeypatch.setenv("INL_SSSP_FRONTIER", "list")
         loop = "graph"
+    elif loop == "graph-trace":
+        trace = tmp_path / "trace.txt"
+        monkeypatch.setenv("INL_SSSP_TRACE", str(trace))
+        monkeypatch.setenv("INL_SSSP_TRACE_MARKS", "1")
+        loop = "graph"
+    elif loop == "dyn-bits":
+        monkeypatch.setenv("INL_SSSP_DYN_BITS", "1")
+        loop = "dyn"
     monkeypatch.setenv("INL_SSSP_LOOP", loop)
     b = inl.bins(flags=inl.BINS_SSSP_DEVLOOP)
     rp, ci, w = csr_from_edges(6, [(1, 2), (2, 3), (3, 1)], [5, 6, 7], symmetric=True)
@@ -118,6 +128,12 @@ def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch):
         assert st["launches"] > 0 and st["host_syncs"] < st0["host_syncs"]
         if loop == "graph":
             assert st["host_syncs"] == 1
+    if trace is not None:  # one block per call; per step: 6 stamps, nF, nsplit, relaxed / marked counters
+        rows = [list(map(int, l.split())) for l in trace.read_text().splitlines() if not l.startswith("#")]
+        assert rows and all(len(r) == 13 for r in rows)
+        last = [r for r in rows if r[1] and r[5]]
+        assert all(r[2] >= r[1] and r[5] >= r[4] for r in last)  # stamps in kernel order
+        assert max(r[11] for r in rows) > 0 and max(r[12] for r in rows) > 0  # relaxed, improved
 
 
 def test_host_buffers(ctx, cfg1):
