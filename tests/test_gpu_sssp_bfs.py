@@ -128,9 +128,9 @@ def test_devloop_edge_cases_and_certificate(ctx, loop, monkeypatch, tmp_path):
         assert st["launches"] > 0 and st["host_syncs"] < st0["host_syncs"]
         if loop == "graph":
             assert st["host_syncs"] == 1
-    if trace is not None:  # one block per call; per step: 6 stamps, nF, nsplit, relaxed / marked counters
+    if trace is not None:  # one block per call; per step: 6 stamps, nF, nsplit, relaxed / marked counters, pieces
         rows = [list(map(int, l.split())) for l in trace.read_text().splitlines() if not l.startswith("#")]
-        assert rows and all(len(r) == 13 for r in rows)
+        assert rows and all(len(r) == 14 for r in rows)
         last = [r for r in rows if r[1] and r[5]]
         assert all(r[2] >= r[1] and r[5] >= r[4] for r in last)  # stamps in kernel order
         assert max(r[11] for r in rows) > 0 and max(r[12] for r in rows) > 0  # relaxed, improved
