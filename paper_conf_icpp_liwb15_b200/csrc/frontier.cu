@@ -936,6 +936,7 @@ __global__ void k_sssp_trace(const SsspDev *s, unsigned long long *tr, int slot,
   unsigned long long *r = tr + step * kTraceSlots;
   r[slot] = t;
   if (slot == 3) r[6] = (unsigned long long)(unsigned)s->nF | ((unsigned long long)(unsigned)s->nsplit << 32);
+  if (slot == 4) r[11] = (unsigned long long)(unsigned)s->gcount;  // grid-bin pieces of the step
   if (slot == 3 || slot == 4) {  // 7 / 8: relaxed / marked after the flat kernel; 9 / 10 after the grid kernel
     r[slot == 3 ? 7 : 9] = *relaxed;
     r[slot == 3 ? 8 : 10] = marks ? *marks : 0ull;
@@ -1816,7 +1817,7 @@ static void sssp_run_graph(inl_ctx ctx, const inl_csr &G, const Bins &b, const u
         fprintf(fp, "%d", i);
         for (int k = 0; k < 6; ++k) fprintf(fp, " %llu", r[k]);
         fprintf(fp, " %u %u", (unsigned)(r[6] & 0xffffffffu), (unsigned)(r[6] >> 32));
-        for (int k = 7; k < 11; ++k) fprintf(fp, " %llu", r[k]);
+        for (int k = 7; k < 12; ++k) fprintf(fp, " %llu", r[k]);
         fprintf(fp, "\n");
       }
       fclose(fp);
