@@ -1242,7 +1242,10 @@ __global__ void __launch_bounds__(256) k_bu_thread(BuArgs a) {
 // vertices of <= kBuThread neighbours) as 4-lane groups (INL_BFS_SMALL=group): 4x fewer L1TEX
 // wavefronts for the column loads than one lane per vertex, but measured no faster (scale 26:
 // 0.47 vs 0.43 ms per launch) — the random frontier-bit probes bound it; k_bu_thread stays.
-constexpr int kBuGroup = 8;
+// lanes per vertex of the warp bin: 2 (4 neighbours per step, 16 vertices per warp) measured
+// best — scale 26: 8 lanes 2.50, 4 lanes 2.35, 2 lanes 2.29, 1 lane 2.33 ms per BFS
+// (profiles/r02/bfs_group_sweep.txt); INL_BFS_GROUP = 1 / 4 / 8 / 16 to measure
+constexpr int kBuGroup = 2;
 constexpr int kBuGroupSpan = 64;
 
 template <int G, int SPAN, bool DEFER>
@@ -2194,8 +2197,26 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
             INL_CUDA(cudaMemsetAsync(f.counts + 3, 0, sizeof(int), st));
             {
               KScope ks(ctx, "k_bu_warp");
-              k_bu_group<kBuGroup, kBuGroupSpan, true><<<grid_for((int64_t)n_large * kBuGroup, ctx->num_sms), 256, 0, st>>>(
-                  ba, deep, f.counts + 3);
+              static int gsz = -1;  // INL_BFS_GROUP: group width of the warp bin (measurement)
+              if (gsz < 0) gsz = getenv("INL_BFS_GROUP") ? atoi(getenv("INL_BFS_GROUP")) : kBuGroup;
+              if (gsz == 1)
+                k_bu_group<1, kBuGroupSpan, true><<<grid_for((int64_t)n_large, ctx->num_sms), 256, 0, st>>>(
+                    ba, deep, f.counts + 3);
+              else if (gsz == 2)
+                k_bu_group<2, kBuGroupSpan, true><<<grid_for((int64_t)n_large * 2, ctx->num_sms), 256, 0, st>>>(
+                    ba, deep, f.counts + 3);
+              else if (gsz == 4)
+                k_bu_group<4, kBuGroupSpan, true><<<grid_for((int64_t)n_large * 4, ctx->num_sms), 256, 0, st>>>(
+                    ba, deep, f.counts + 3);
+              else if (gsz == 8)
+                k_bu_group<8, kBuGroupSpan, true><<<grid_for((int64_t)n_large * 8, ctx->num_sms), 256, 0, st>>>(
+                    ba, deep, f.counts + 3);
+              else if (gsz == 16)
+                k_bu_group<16, kBuGroupSpan, true><<<grid_for((int64_t)n_large * 16, ctx->num_sms), 256, 0, st>>>(
+                    ba, deep, f.counts + 3);
+              else
+                k_bu_group<kBuGroup, kBuGroupSpan, true><<<grid_for((int64_t)n_large * kBuGroup, ctx->num_sms), 256, 0,
+                                                            st>>>(ba, deep, f.counts + 3);
             }
             KScope ks(ctx, "k_bu_deep");
             k_bu_deep<<<ctx->num_sms * 2, 256, 0, st>>>(ba, deep, f.counts + 3);
