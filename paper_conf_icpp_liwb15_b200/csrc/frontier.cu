@@ -2131,7 +2131,12 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
       if (nF == 0) break;
       // Beamer's switch: enter bottom-up when the frontier's edges exceed the unvisited
       // edges / 14 (or it holds > n/24 vertices), leave it below n/256 vertices
-      const bool want_bu = allow_bu && (bu ? nF > n / 256 : (nF > n / 24 || (double)mf_next * 14.0 > (double)m_u));
+      static double alpha = -1.0, beta = -1.0;  // Beamer's alpha (14) and beta (24); INL_BFS_AB=a,b to measure
+      if (alpha < 0.0) {
+        alpha = 14.0, beta = 24.0;
+        if (const char *e = getenv("INL_BFS_AB")) sscanf(e, "%lf,%lf", &alpha, &beta);
+      }
+      const bool want_bu = allow_bu && (bu ? nF > n / 256 : (nF > (int64_t)(n / beta) || (double)mf_next * alpha > (double)m_u));
       if (want_bu) {
         if (queue_ok) {  // frontier queue -> bitmap
           INL_CUDA(cudaMemsetAsync(fa, 0, sizeof(uint32_t) * nwords, st));
