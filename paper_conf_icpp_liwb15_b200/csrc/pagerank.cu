@@ -55,6 +55,26 @@ __global__ void __launch_bounds__(1024) k_pr_dsum(const double *__restrict__ dpa
   }
 }
 
+// Stage 1 of the fixed-order dangling sum for large m: CTA b sums the b-th contiguous chunk of
+// the partials (the same tree as k_pr_dsum) into part[b]; k_pr_dsum then adds the part[] in
+// order.  Deterministic for a given m and grid; one CTA alone took 43 us at scale 25.
+__global__ void __launch_bounds__(1024) k_pr_dsum_part(const double *__restrict__ dpart, int64_t m,
+                                                       double *__restrict__ part) {
+  __shared__ double red[32];
+  const int64_t per = (m + gridDim.x - 1) / gridDim.x;
+  const int64_t lo = blockIdx.x * per, hi = min(m, lo + per);
+  double s = 0.0;
+  for (int64_t i = lo + threadIdx.x; i < hi; i += 1024) s += dpart[i];
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int i = 0; i < 32; ++i) t += red[i];
+    part[blockIdx.x] = t;
+  }
+}
+
 // D = sum over ranks in rank order; base = (1-d)/n + d*D/n.
 __global__ void k_pr_base(const double *__restrict__ dall, int nranks, int64_t n, double d,
                           float *__restrict__ base) {
@@ -395,11 +415,23 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
   INL_CUDA(cudaMemsetAsync(c_cur, 0, sizeof(float) * ncomp, st));
   INL_CUDA(cudaMemsetAsync(c_next, 0, sizeof(float) * ncomp, st));
   const int32_t *cidx = (const int32_t *)p->pr_cidx.p;
-  char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (P + 1));
+  constexpr int kDsumParts = 1024;  // stage-1 partials of the dangling sum (<= num_sms CTAs)
+  char *scal = (char *)ctx->s_c.get(256 + sizeof(double) * (P + 1 + kDsumParts));
   float *base = (float *)scal;
   unsigned long long *ndang = (unsigned long long *)(scal + 8);
   double *dloc = (double *)(scal + 16);
   double *dall = (double *)(scal + 256);
+  double *dparts = dall + P + 1;
+  // fixed-order dangling sum of m partials: one CTA for small m, else stage 1 over G CTAs first
+  auto dsum = [&](const double *src, int64_t cnt, double *out) {
+    const int G = (int)std::min<int64_t>(std::min(ctx->num_sms, kDsumParts), cnt / 8192);
+    if (G > 1) {
+      k_pr_dsum_part<<<G, 1024, 0, st>>>(src, cnt, dparts);
+      k_pr_dsum<<<1, 1024, 0, st>>>(dparts, G, out);
+    } else {
+      k_pr_dsum<<<1, 1024, 0, st>>>(src, cnt, out);
+    }
+  };
   float *rank_pad = nullptr;
   if (DIST) rank_pad = (float *)ctx->s_d.get(sizeof(float) * npad);
 
@@ -424,7 +456,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
     if (K == 1) {
       launch_gather<false>(ctx, p, a, epi, dpart, (const int32_t *)p->pr_col.p, pr_hot, &p->pr_cb, p->pr_nhot);
       if (!last) {
-        k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, DIST ? dloc : dall);
+        dsum(dpart, m, DIST ? dloc : dall);
         INL_CUDA(cudaGetLastError());
         if (DIST) comm_allgather(ctx, c_next + (int64_t)ctx->rank * Bc, c_next, Bc, ncclFloat32, dloc, dall);
       }
@@ -448,7 +480,7 @@ void pagerank_run(inl_ctx ctx, inl_plan p, const int32_t *out_degree, float damp
         }
       }
       if (!last) {
-        k_pr_dsum<<<1, 1024, 0, st>>>(dpart, m, dloc);
+        dsum(dpart, m, dloc);
         INL_CUDA(cudaGetLastError());
         cudaEvent_t ev = ctx_event(ctx, 1);
         INL_CUDA(cudaEventRecord(ev, st));
