@@ -1,3 +1,5 @@
+# Experiment record: INL_SSSP_CARVEOUT (a uniform smem carveout for the SSSP loop kernels) was measured
+# slower at every setting and removed from frontier.cu; this script no longer changes anything.
 mkdir -p gpurun_out
 B="python bench.py --no-e2e --no-cpu-baseline --no-context --op sssp --steps 9 --warmup 3"
 o=gpurun_out/ab_carveout.txt; : > $o

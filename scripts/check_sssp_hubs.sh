@@ -1,3 +1,5 @@
+# Experiment record: the hub-deferral code (INL_SSSP_HUBS) measured 2.1x slower and was not kept
+# (profiles/r02/sssp_hub_deferral_experiment.txt); the INL_SSSP_HUBS switch no longer exists.
 mkdir -p gpurun_out
 B="python bench.py --no-e2e --no-cpu-baseline --no-context --op sssp --steps 9 --warmup 3"
 o=gpurun_out/check_hubs.txt; : > $o
