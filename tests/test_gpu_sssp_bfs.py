@@ -240,3 +240,30 @@ def test_dbuf_global_template_default_t_block(ctx, lbt):
     wb = inlgen.weights_host(rp, ci)
     d, _ = gpu_sssp(ctx, rp, ci, wb, len(rp) - 1, 0, b)
     assert np.array_equal(d, oracle.sssp(rp, ci, wb, 0))
+
+
+def test_bfs_bottom_up_entered_twice(ctx):
+    """Two dense clusters joined by a long path: BFS goes bottom-up in the first cluster,
+    top-down along the path, and bottom-up again in the second — the second entry starts from
+    the plan's static degree bins, most of whose vertices (the first cluster) are visited and
+    must be skipped.  Levels bit-exact against the oracle, with the direction switches taken."""
+    rng = np.random.default_rng(7)
+    na, npath = 6000, 120
+    n = 2 * na + npath
+    e = set()
+    for base in (0, na + npath):  # two clusters: random graph, mean degree ~24, plus a few hubs
+        for _ in range(na * 12):
+            u, v = rng.integers(0, na, 2)
+            if u != v:
+                e.add((base + int(min(u, v)), base + int(max(u, v))))
+        for h in range(8):
+            for v in rng.choice(na, 400, replace=False):
+                if int(v) != h:
+                    e.add((base + min(h, int(v)), base + max(h, int(v))))
+    chain = [na - 1] + list(range(na, na + npath)) + [na + npath]
+    e.update((a, b) for a, b in zip(chain[:-1], chain[1:]))
+    rp, ci, _ = csr_from_edges(n, sorted(e), symmetric=True)
+    for s in (0, 17, n - 1):
+        lv, st = gpu_bfs(ctx, rp, ci, n, s, inl.bins())
+        assert np.array_equal(lv, oracle.bfs(rp, ci, s))
+        assert st["iterations"] > npath
