@@ -230,7 +230,8 @@ inl_status inl_pagerank(inl_ctx ctx, const inl_csr *A_in, const int32_t *out_deg
                         int32_t iterations, float *rank, inl_plan plan);
 
 /* SSSP (P5@10241, P11@2218): frontier Bellman-Ford relaxation (atomicMin) until no distance
- * changes (one GPU: near-far scheduled, the step loop as one CUDA-graph launch).  w [nnz]
+ * changes (one GPU: near-far scheduled with bitmap frontiers, the step loop as one CUDA-graph
+ * launch).  w [nnz]
  * uint32 >= 1, dist [n_global] uint32 with UINT32_MAX = unreachable (replicated).  Distances
  * must stay < 2^32 - 2^8.  Blocks until converged. */
 inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t source,
@@ -238,7 +239,9 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
 
 /* BFS (P5@11591): level-synchronous frontier expansion (one GPU: direction-optimizing when the
  * plan found the graph symmetric, bottom-up levels over degree-binned worklists of the unvisited
- * vertices); level [n_global] int32, -1 = unreachable, level[source] = 0 (replicated).
+ * vertices — the first bottom-up level reads the plan's static degree bins, which a symmetric
+ * plan builds at creation: 4 B per vertex of degree > 0 in the plan's memory); level
+ * [n_global] int32, -1 = unreachable, level[source] = 0 (replicated).
  * Blocks until converged. */
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
                    inl_stats *stats, inl_plan plan);
