@@ -240,7 +240,7 @@ inl_status inl_sssp(inl_ctx ctx, const inl_csr *G, const uint32_t *w, int64_t so
 /* BFS (P5@11591): level-synchronous frontier expansion (one GPU: direction-optimizing when the
  * plan found the graph symmetric, bottom-up levels over degree-binned worklists of the unvisited
  * vertices — the first bottom-up level reads the plan's static degree bins, which a symmetric
- * plan builds at creation: 4 B per vertex of degree > 0 in the plan's memory); level
+ * plan builds at creation: 8 B per vertex in the plan's memory); level
  * [n_global] int32, -1 = unreachable, level[source] = 0 (replicated).
  * Blocks until converged. */
 inl_status inl_bfs(inl_ctx ctx, const inl_csr *G, int64_t source, int32_t *level,
