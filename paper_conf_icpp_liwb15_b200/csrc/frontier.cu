@@ -593,7 +593,10 @@ __global__ void __launch_bounds__(NT) k_expand(ExpandArgs a, Op op) {
 // consecutive edges of the window (one upper-bound search per window, then a walk),
 // so all threads do equal work and a warp touches consecutive edges.  Vertices of
 // larger degree go to the global grid buffer (dbuf-global) as grid_chunk pieces.
-constexpr int kEdgesPerThread = 8;
+#ifndef INL_EPT
+#define INL_EPT 8
+#endif
+constexpr int kEdgesPerThread = INL_EPT;  // edges in flight per thread in the expansion kernels
 
 template <class Op>
 __global__ void __launch_bounds__(NT, INL_EXPAND_MINB) k_expand_flat(ExpandArgs a, Op op) {
