@@ -5,7 +5,6 @@
 #include <stdint.h>
 
 #include <string>
-#include <utility>
 #include <cstdlib>
 #include <vector>
 
@@ -236,35 +235,6 @@ struct KScope {
     sl->pending.emplace_back(e0, e1);
   }
 };
-// Whether PDL launches are on (INL_PDL=0 turns them off, for A/B measurement).
-inline bool pdl_enabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("INL_PDL");
-    v = e ? atoi(e) != 0 : 1;
-  }
-  return v == 1;
-}
-
-// Launch `k` on ctx's stream with a programmatic dependency on the previous kernel of the stream
-// (cudaLaunchAttributeProgrammaticStreamSerialization): its CTAs may launch while that kernel
-// drains, and must call pdl_wait() before touching anything the previous kernel writes or reads.
-template <typename... KArgs, typename... Args>
-cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
-                       Args &&...args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = st;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
-}
-
 // plan.cu
 void build_plan(inl_plan p);
 // spmv.cu
