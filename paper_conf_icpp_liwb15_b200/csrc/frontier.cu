@@ -242,6 +242,11 @@ struct BfsOp {
   // NEXT-1 fused exchange (DIST): a discovered vertex v sets its bit in the next-frontier
   // bitmap of its OWNER q = v / B, in q's memory (NVLink peer memory; the same device for the
   // loopback), during the expansion itself — no byte map, no allreduce
+  // one-GPU top-down with fire-and-forget marks: a candidate sets its visited bit and its bit
+  // in nbits (the next frontier) with red.or and stores level L+1 (every discoverer stores the
+  // same value) — no returning atomicOr, no queue push; k_bfs_next_queue builds the queue and
+  // m_f from nbits afterwards
+  uint32_t *nbits = nullptr;
   uint32_t *const *xtab = nullptr;   // [P] owners' bitmaps of this level
   int64_t B = 0;                     // row block
   const uint32_t *xself = nullptr;   // this rank's own bitmap (local sets are not exchange)
@@ -285,6 +290,17 @@ struct BfsOp {
 #pragma unroll
     for (int j = 0; j < K; ++j)
       if (!((bw[j] >> (vv[j] & 31)) & 1u)) cand |= 1u << j;
+    if (nbits) {
+#pragma unroll
+      for (int j = 0; j < K; ++j)
+        if ((cand >> j) & 1u) {
+          const uint32_t bit = 1u << (vv[j] & 31);
+          red_or_b32(bitmap + (vv[j] >> 5), bit);
+          red_or_b32(nbits + (vv[j] >> 5), bit);
+          level[vv[j]] = L + 1;
+        }
+      return;
+    }
     if (!enqueue) {
       if (xtab) {
         unsigned rem = 0;
@@ -1357,6 +1373,35 @@ __global__ void k_queue_to_bitmap(const int32_t *__restrict__ q, int nq, uint32_
     atomicOr(bm + (q[i] >> 5), 1u << (q[i] & 31));
 }
 
+// next frontier bitmap -> queue (one counter atomic per warp) and its degree sum (Beamer's m_f)
+__global__ void k_bfs_next_queue(const uint32_t *__restrict__ nb, int64_t nwords, const int64_t *__restrict__ rp,
+                                 int32_t *q, int *cnt, unsigned long long *mf) {
+  const int64_t nr = (nwords + 31) / 32 * 32;  // whole warps iterate together
+  const int lane = threadIdx.x & 31;
+  unsigned long long dg = 0;
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nr; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t b = w < nwords ? nb[w] : 0u;
+    if (!__any_sync(0xffffffffu, b != 0u)) continue;
+    const int c = __popc(b);
+    int incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
+    int base = 0;
+    if (lane == 31) base = atomicAdd(cnt, incl);
+    int pos = __shfl_sync(0xffffffffu, base, 31) + incl - c;
+    for (; b; b &= b - 1) {
+      const int32_t v = (int32_t)(w * 32 + __ffs(b) - 1);
+      q[pos++] = v;
+      dg += (unsigned long long)(rp[v + 1] - rp[v]);
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) dg += __shfl_xor_sync(0xffffffffu, dg, o);
+  if (lane == 0 && dg) atomicAdd(mf, dg);
+}
+
 __global__ void k_bitmap_to_queue(const uint32_t *__restrict__ bm, int64_t n, int32_t *q, int *cnt) {
   const int64_t nwords = (n + 31) / 32;
   for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nwords;
@@ -2086,12 +2131,20 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   // direction optimisation (Beamer et al.): bottom-up while the frontier holds more than
   // n / kBuEnter vertices, top-down again once it falls below n / kBuLeave
   const int64_t nwords = (n + 31) / 32;
-  uint32_t *fa = nullptr, *fb = nullptr;
+  uint32_t *fa = nullptr, *fb = nullptr, *tdb = nullptr;  // tdb: top-down next-frontier bitmap
   bool bu = false;       // direction of the previous step
   bool queue_ok = true;  // f.F holds the frontier (else the bitmap fa does)
   // bottom-up scans a vertex's row for frontier parents: valid only when rows list the
   // predecessors too (a symmetric graph, verified by the plan)
   const bool allow_bu = symmetric && !(b.flags & (INL_BINS_THREAD_ONLY | kTemplateFlags)) && n >= 4096;
+  // top-down steps with fire-and-forget marks (BfsOp::nbits) where the flat / grid kernels run
+  // (INL_BFS_TD=atomic keeps the claim-by-atomicOr queue pushes, for A/B)
+  static int td_env = -1;
+  if (td_env < 0) {
+    const char *e = getenv("INL_BFS_TD");
+    td_env = e && std::string(e) == "atomic" ? 0 : 1;
+  }
+  const bool td_red = allow_bu && td_env == 1 && expand_cfg(G, b).flat;
   // Beamer's m_f (degree sum of the next frontier) and m_u (edges of unvisited vertices)
   unsigned long long *mfp = (unsigned long long *)(f.counts + 10);
   unsigned long long mf_next = 0;
@@ -2118,7 +2171,8 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
   int n_small = 0, n_large = 0, bl_cur = 0;
   bool lists_ok = false;  // the worklists hold exactly the unvisited vertices of degree > 0
   if (allow_bu) {
-    fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 2 * (nwords + 1));
+    fa = (uint32_t *)ctx->s_g.get(sizeof(uint32_t) * 3 * (nwords + 1));
+    tdb = fa + 2 * (nwords + 1);  // fixed: fa / fb swap roles every bottom-up level
     fb = fa + nwords + 1;
     if (!bu_word) {
       int32_t *L4 = (int32_t *)ctx->s_bu.get(sizeof(int32_t) * 4 * (size_t)(n + 1));
@@ -2260,7 +2314,20 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
         lists_ok = false;  // top-down visits vertices the worklists still hold
         BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, allow_bu ? mfp : nullptr};  // m_f only when it decides
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
-        expand(ctx, G, b, f, nF, op);
+        // fire-and-forget marks pay for their bitmap clear + scan only on a heavy level (edges
+        // of the frontier > nnz / 64: scale 26 2.30 -> 2.10 ms per BFS; on every level scale 23
+        // lost 4%; profiles/r02/bfs_td_marks.txt)
+        if (td_red && (double)mf_next * 64.0 > (double)G.nnz) {
+          uint32_t *nb = tdb;
+          INL_CUDA(cudaMemsetAsync(nb, 0, sizeof(uint32_t) * nwords, st));
+          op.nbits = nb;
+          op.mf = nullptr;
+          expand(ctx, G, b, f, nF, op);  // clears the queue counter; no pushes
+          k_bfs_next_queue<<<grid_for(nwords, ctx->num_sms), 256, 0, st>>>(nb, nwords, G.row_ptr, f.Fout, f.counts, mfp);
+          INL_CUDA(cudaGetLastError());
+        } else {
+          expand(ctx, G, b, f, nF, op);
+        }
         read_level(&nF, &mf_next);
         std::swap(f.F, f.Fout);
         queue_ok = true;
