@@ -2315,9 +2315,12 @@ void bfs_run(inl_ctx ctx, const inl_csr &G, const Bins &b, int64_t source, int32
         BfsOp op{bm, level, nullptr, n, L, true, 0, G.row_ptr, allow_bu ? mfp : nullptr};  // m_f only when it decides
         INL_CUDA(cudaMemsetAsync(mfp, 0, sizeof(unsigned long long), st));
         // fire-and-forget marks pay for their bitmap clear + scan only on a heavy level (edges
-        // of the frontier > nnz / 64: scale 26 2.30 -> 2.10 ms per BFS; on every level scale 23
-        // lost 4%; profiles/r02/bfs_td_marks.txt)
-        if (td_red && (double)mf_next * 64.0 > (double)G.nnz) {
+        // of the frontier > nnz / 256: scale 26 2.30 -> 2.02 ms per BFS, the heaviest level
+        // 1.70 -> 0.48 ms; on every level scale 23 lost 4%; divisors 16 / 64 / 256 / 1024:
+        // profiles/r02/bfs_td_marks.txt); INL_BFS_TD_DIV to measure
+        static double td_div = -1.0;
+        if (td_div < 0.0) td_div = getenv("INL_BFS_TD_DIV") ? atof(getenv("INL_BFS_TD_DIV")) : 256.0;
+        if (td_red && (double)mf_next * td_div > (double)G.nnz) {
           uint32_t *nb = tdb;
           INL_CUDA(cudaMemsetAsync(nb, 0, sizeof(uint32_t) * nwords, st));
           op.nbits = nb;
