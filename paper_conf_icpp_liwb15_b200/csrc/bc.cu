@@ -22,6 +22,7 @@
 #include <vector>
 
 #include "inl_internal.cuh"
+#include "ptx.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -61,6 +62,9 @@ struct BcArgs {
   int32_t source;
   BcPk *pk;
   int32_t tag;
+  // heavy push levels: claims are plain level stores + a fire-and-forget bit in nbits (no
+  // returning atomicCAS, no queue counter); k_bc_bits_to_q appends the level in vertex order
+  uint32_t *nbits = nullptr;
 };
 
 // append v to level L+1 (one counter atomic per coalesced group)
@@ -70,6 +74,28 @@ __device__ __forceinline__ void enqueue(const BcArgs &a, int32_t v) {
   if (g.thread_rank() == 0) pos = atomicAdd(a.qcount, (int)g.size());
   pos = g.shfl(pos, 0) + (int)g.thread_rank();
   a.Q[a.hi + pos] = v;
+}
+
+// the level claimed through nbits -> Q[hi, hi + count) in vertex order, count in *qcount (one
+// counter atomic per warp)
+__global__ void k_bc_bits_to_q(const uint32_t *__restrict__ nb, int64_t nwords, int32_t *Qn, int *qcount) {
+  const int64_t nr = (nwords + 31) / 32 * 32;
+  const int lane = threadIdx.x & 31;
+  for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < nr; w += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t b = w < nwords ? nb[w] : 0u;
+    if (!__any_sync(0xffffffffu, b != 0u)) continue;
+    const int c = __popc(b);
+    int incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
+    int base = 0;
+    if (lane == 31) base = atomicAdd(qcount, incl);
+    int pos = __shfl_sync(0xffffffffu, base, 31) + incl - c;
+    for (; b; b &= b - 1) Qn[pos++] = (int32_t)(w * 32 + __ffs(b) - 1);
+  }
 }
 
 // m_f of the level just built: degree sum of Q[hi, hi + *qcount) (Beamer's frontier edge
@@ -89,8 +115,13 @@ __global__ void k_bc_degsum(BcArgs a) {
 __device__ __forceinline__ void fwd_edge(const BcArgs &a, double su, int32_t v) {
   int lv = a.level[v];
   if (lv == -1) {
-    const int old = atomicCAS(a.level + v, -1, a.L + 1);
-    if (old == -1) enqueue(a, v);
+    if (a.nbits) {  // every discoverer stores the same level; the bitmap deduplicates
+      a.level[v] = a.L + 1;
+      red_or_b32(a.nbits + (v >> 5), 1u << (v & 31));
+    } else {
+      const int old = atomicCAS(a.level + v, -1, a.L + 1);
+      if (old == -1) enqueue(a, v);
+    }
     lv = a.L + 1;  // whoever won, only level L+1 is claimed in this step
   }
   if (lv == a.L + 1) atomicAdd(a.sigma + v, su);
@@ -670,6 +701,16 @@ void bc_src_run(inl_ctx ctx, const inl_csr &G, const int64_t *sources, int64_t n
 
 }  // namespace
 
+// fire-and-forget claims on heavy push levels (INL_BC_MARKS=0 keeps atomicCAS + queue pushes)
+static bool bc_marks() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("INL_BC_MARKS");
+    v = e ? atoi(e) != 0 : 1;
+  }
+  return v == 1;
+}
+
 void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources, int64_t n_sources, double *bc,
             inl_stats *stats, bool symmetric) {
   cudaStream_t st = ctx->stream;
@@ -693,6 +734,8 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources
   double *bigpart = (double *)ctx->s_g.get(sizeof(double) * maxp);
   int4 *bigv = (int4 *)ctx->s_tmp.get(sizeof(int4) * (G.nnz / kBcWarp + 16));
   int *cnt = (int *)ctx->s_f.get(64);  // [0] queue [1] pieces [2] large vertices; m_f at byte 16
+  const int64_t nwb = (n + 31) / 32;
+  uint32_t *nbits = (uint32_t *)ctx->s_bcb.get(sizeof(uint32_t) * (nwb + 1));
   unsigned long long *mfp = (unsigned long long *)(cnt + 4);
   k_zero_d<<<grid_of(n, ctx->num_sms), 256, 0, st>>>(bc, n);
   INL_CUDA(cudaGetLastError());
@@ -777,9 +820,20 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources
         launches += 1;
       } else {
         KScope ks(ctx, "k_bc_fwd");
+        // heavy push level (frontier edges > nnz / 256): fire-and-forget claims, see BcArgs::nbits
+        const bool marks = bc_marks() && (double)mf_next * 256.0 > (double)G.nnz;
+        if (marks) {
+          a.nbits = nbits;
+          INL_CUDA(cudaMemsetAsync(nbits, 0, sizeof(uint32_t) * nwb, st));
+        }
         k_bc_level<true><<<(a.hi - a.lo + kBcNT - 1) / kBcNT, kBcNT, 0, st>>>(a);
         k_bc_big<true><<<ctx->num_sms * 4, kBcNT, 0, st>>>(a);
         launches += 2;
+        if (marks) {
+          k_bc_bits_to_q<<<grid_of(nwb, ctx->num_sms), 256, 0, st>>>(nbits, nwb, Q + a.hi, cnt);
+          ++launches;
+          a.nbits = nullptr;
+        }
       }
       if (pull_edge > 0.0 && !tpl) {
         k_bc_degsum<<<ctx->num_sms * 2, 256, 0, st>>>(a);

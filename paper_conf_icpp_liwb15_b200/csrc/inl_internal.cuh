@@ -156,6 +156,7 @@ struct inl_ctx_s {
   inl::DevBuf s_bu;                                    // BFS bottom-up worklists
   inl::DevBuf s_h;                                     // tree levels (tree.cu)
   inl::DevBuf s_t;                                     // SSSP step trace (INL_SSSP_TRACE, measurement)
+  inl::DevBuf s_bcb;                                   // BC next-level bitmap (heavy push levels)
   int64_t *pinned = nullptr;                           // small pinned host scalars
   int live_plans = 0;    // plans created on this ctx and not yet destroyed
   struct inl_plan_s *tplan = nullptr;  // reusable transient plan (plan = NULL calls)
