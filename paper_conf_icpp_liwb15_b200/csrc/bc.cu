@@ -866,7 +866,7 @@ void bc_run(inl_ctx ctx, const inl_csr &G, const Bins &b, const int64_t *sources
         KScope ks(ctx, "k_bc_bwd");
         k_bc_level<false><<<(a.hi - a.lo + kBcNT - 1) / kBcNT, kBcNT, 0, st>>>(a);
         k_bc_big<false><<<ctx->num_sms * 4, kBcNT, 0, st>>>(a);
-        k_bc_combine<<<8, 128, 0, st>>>(a);
+        k_bc_combine<<<ctx->num_sms * 4, 128, 0, st>>>(a);  // one thread per large vertex (8 CTAs: 256 us at scale 22)
       }
       launches += 3;
       INL_CUDA(cudaGetLastError());
